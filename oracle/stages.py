@@ -1,0 +1,86 @@
+"""The staged decomposition the GPU path uses, written plainly (test infrastructure only).
+
+This is the oracle for stage-level parity: every intermediate here is a unique
+group element (or integer) once the window size c and the digit rule are fixed,
+so the GPU's bucket sums and window sums can be compared one by one.
+
+Signed-digit rule (PAPER.md:428 adopts signed digits without stating a rule;
+DESIGN.md reading R6):
+    nwin = floor(λ / c) + 1
+    chunk_j = bits [j c, j c + c) of k;  d_j = chunk_j + carry_j
+    for j < nwin-1: if d_j > 2^(c-1): d_j -= 2^c, carry_{j+1} = 1 else carry_{j+1} = 0
+    the top digit is never negated.
+    => k = sum_j d_j 2^(j c), d_j in (-2^(c-1), 2^(c-1)] (top digit in [0, 2^(c-1)]).
+Bucket of a digit: |d_j| in [0, 2^(c-1)] (0 = no bucket), sign = d_j < 0 (the point
+is negated, y -> p - y).
+
+B_{j,b} = sum_{i : |d_ij| = b} sgn(d_ij) P_i                 (bucket-sum)
+W_j     = sum_{b=1}^{2^(c-1)} b * B_{j,b}                     (bucket-reduce, PAPER.md:143, 161;
+                                                             "2^i B_i" read as b*B_b, R12)
+Q       = sum_j 2^(j c) W_j  by Horner                        (window-reduce)
+"""
+from . import ec
+
+
+def num_windows(lam: int, c: int) -> int:
+    return lam // c + 1
+
+
+def signed_digits(k: int, lam: int, c: int) -> list[int]:
+    assert 0 <= k < (1 << lam)
+    nwin = num_windows(lam, c)
+    half = 1 << (c - 1)
+    mask = (1 << c) - 1
+    out = []
+    carry = 0
+    for j in range(nwin):
+        d = ((k >> (j * c)) & mask) + carry
+        if j < nwin - 1 and d > half:
+            d -= 1 << c
+            carry = 1
+        else:
+            carry = 0
+        out.append(d)
+    return out
+
+
+def bucket_sums(ks, Ps, c, curve):
+    """Returns B[j][b] (affine, None = O) for b in 0..2^(c-1) (B[j][0] unused = None)."""
+    nwin = num_windows(curve.lam, c)
+    nb = (1 << (c - 1)) + 1
+    B = [[None] * nb for _ in range(nwin)]
+    for k, P in zip(ks, Ps):
+        ds = signed_digits(k, curve.lam, c)
+        for j, d in enumerate(ds):
+            if d == 0:
+                continue
+            Q = P if d > 0 else ec.neg(P, curve)
+            B[j][abs(d)] = ec.add(B[j][abs(d)], Q, curve)
+    return B
+
+
+def window_sums(B, curve):
+    """W_j = sum_b b * B_{j,b}, by the descending running sum."""
+    W = []
+    for Bj in B:
+        running = None
+        Wj = None
+        for b in range(len(Bj) - 1, 0, -1):
+            running = ec.add(running, Bj[b], curve)
+            Wj = ec.add(Wj, running, curve)
+        W.append(Wj)
+    return W
+
+
+def window_combine(W, c, curve):
+    """Q = sum_j 2^(j c) W_j by Horner: c PDBL per window step."""
+    Q = None
+    for j in range(len(W) - 1, -1, -1):
+        for _ in range(c):
+            Q = ec.double(Q, curve)
+        Q = ec.add(Q, W[j], curve)
+    return Q
+
+
+def msm_staged(ks, Ps, c, curve):
+    return window_combine(window_sums(bucket_sums(ks, Ps, c, curve), curve), c, curve)
