@@ -1,0 +1,385 @@
+#!/usr/bin/env python3
+"""bench.py — MSM latency / throughput of the B200 library on BASELINE.json's headline
+workload (default: BLS12-381 G1, n = 2^26, config C4), one JSON line on rank 0.
+
+    python bench.py [--gpus N] [--steps K] [--warmup W] [--curve C] [--log2n L] [--impl reference]
+
+N = 1: one process, one context on cuda:0.  N > 1 (launched by torchrun, one process per
+GPU, NCCL): the n points are split into N contiguous shards (strong scaling: total n fixed);
+each rank computes its partial MSM (msm_run_partial), the partials are all-gathered over
+NCCL and rank 0 adds them (msm_finalize).  A "step" is one whole MSM of n points.
+
+Timing: W untimed warm-ups; K timed steps between a barrier + cuda.synchronize on both
+sides; CUDA events on the library's stream; max over ranks.  The inputs (points 112 B x n,
+scalars 32 B x n) exceed the 126 MB L2 many times, so no explicit flush is needed.
+"""
+import argparse
+import json
+import os
+import statistics
+import subprocess
+import sys
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+CURVE_INFO = {  # name: (L32, S, lambda, L (radix-2^W limbs), W)
+    "bn254": (8, 8, 254, 9, 30),
+    "bls12_377": (12, 8, 253, 13, 30),
+    "bls12_381": (12, 8, 255, 13, 30),
+    "mnt4_753": (24, 24, 753, 27, 29),
+}
+METRIC = "MSM latency (ms) and points/sec at 2^20–2^26, 1/2/4/8 B200; % IMAD roofline"
+PAPER_MS = {("bls12_381", 26, 1): 855.2, ("bls12_381", 26, 8): 113.7, ("bls12_377", 24, 1): 213.6,
+            ("bls12_377", 24, 8): 30.35, ("mnt4_753", 22, 1): 863.8, ("mnt4_753", 22, 8): 116.8}
+
+
+def imad_slots_per_mult(L):
+    """IMAD-pipe issue slots of one radix-2^W Montgomery multiplication as implemented:
+    2L^2 limb products as IMAD.WIDE.U32 (2 slots each on sm_100a: half rate, measured in
+    microbench/imad_peak.cu) + L low-only IMAD for m_k = t_k n'_0 (1 slot)."""
+    return 2 * L * L * 2 + L
+
+
+def peaks():
+    path = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    try:
+        return json.load(open(path))
+    except Exception:
+        return {"hbm_gbs": 6650.0, "sm_max_mhz": 1965.0, "fallback": True}
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+
+    FIELDS = ("clocks.sm,clocks.max.sm,power.draw,clocks_event_reasons.active,"
+              "clocks_event_reasons.hw_slowdown,clocks_event_reasons.hw_thermal_slowdown,"
+              "clocks_event_reasons.sw_thermal_slowdown,clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, index):
+        self.index = index
+        self.rows = []
+        self._stop = threading.Event()
+        self._t = None
+
+    def _run(self):
+        while not self._stop.is_set():
+            try:
+                out = subprocess.run(["nvidia-smi", "-i", str(self.index), "--query-gpu=" + self.FIELDS,
+                                      "--format=csv,noheader,nounits"], capture_output=True, text=True, timeout=5)
+                if out.returncode == 0 and out.stdout.strip():
+                    self.rows.append([v.strip() for v in out.stdout.strip().split(",")])
+            except Exception:
+                pass
+            self._stop.wait(0.2)
+
+    def __enter__(self):
+        self._t = threading.Thread(target=self._run, daemon=True)
+        self._t.start()
+        return self
+
+    def __exit__(self, *a):
+        self._stop.set()
+        self._t.join(timeout=10)
+
+    def summary(self):
+        if not self.rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["unavailable"], "samples": 0}
+        sm = [float(r[0]) for r in self.rows if r[0].replace(".", "").isdigit()]
+        mx = [float(r[1]) for r in self.rows if r[1].replace(".", "").isdigit()]
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in self.rows for i in range(4) if len(r) > 4 + i and r[4 + i] == "Active"})
+        return {"sm_mhz": statistics.median(sm) if sm else None, "sm_max_mhz": max(mx) if mx else None,
+                "reasons": reasons, "samples": len(self.rows),
+                "power_w_max": max((float(r[2]) for r in self.rows if r[2].replace(".", "").isdigit()), default=None)}
+
+
+def dist_env():
+    ws = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    return ws, rank, local
+
+
+# ---------------------------------------------------------------------------------------
+def cpu_baseline(curve, seconds_hint=True, n_sample=None):
+    """The oracle's plain Pippenger as it stands, single process, on a
+    bounded sample of the same workload (same curve, same input recipe)."""
+    import synth
+    from oracle import msm as omsm, points as opoints
+    from oracle.curves import CURVES
+    c = CURVES[curve]
+    if n_sample is None:
+        n_sample = 1 << 11 if curve != "mnt4_753" else 1 << 8
+    e0, d = synth.point_seeds(c.r, 20240427)
+    Ps = opoints.progression_points(e0, d, n_sample, c)
+    ks = synth.words_to_ints(synth.scalars_range(c.r, 0, n_sample, 20240427))
+    t0 = time.perf_counter()
+    omsm.msm_pippenger(ks, Ps, c, s=8)
+    dt = time.perf_counter() - t0
+    return {"value": n_sample / dt, "unit": "points/s", "cores": 1, "kind": "oracle",
+            "sample": f"{curve} n={n_sample} (first {n_sample} points/scalars of the workload recipe), "
+                      f"oracle.msm_pippenger s=8, pure-Python ints, 1 process; {dt:.2f} s",
+            "seconds": dt}
+
+
+def run_reference(args):
+    ws, rank, local = dist_env()
+    if rank != 0:
+        return 0
+    curve = args.curve
+    n_sample = args.ref_sample or (1 << 10 if curve != "mnt4_753" else 1 << 7)
+    import synth
+    from oracle import msm as omsm, points as opoints
+    from oracle.curves import CURVES
+    c = CURVES[curve]
+    e0, d = synth.point_seeds(c.r, 20240427)
+    Ps = opoints.progression_points(e0, d, n_sample, c)
+    ks = synth.words_to_ints(synth.scalars_range(c.r, 0, n_sample, 20240427))
+    for _ in range(args.warmup):
+        omsm.msm_pippenger(ks, Ps, c, s=8)
+    times = []
+    for _ in range(args.steps):
+        t0 = time.perf_counter()
+        omsm.msm_pippenger(ks, Ps, c, s=8)
+        times.append(time.perf_counter() - t0)
+    ms = statistics.median(times) * 1e3
+    val = n_sample / (ms / 1e3)
+    line = {
+        "impl": "reference", "metric": METRIC, "value": val, "unit": "points/s", "n_gpus": args.gpus,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
+        "scaling": "strong", "vs_baseline": None, "dtype": "int (python big ints)", "data": "synthetic",
+        "config": {"workload": f"{curve} G1 MSM n=2^{args.log2n}", "curve": curve, "n": 1 << args.log2n,
+                   "sample_n": n_sample, "l2": "n/a (CPU)"},
+        "cpu_baseline": {"value": val, "unit": "points/s", "cores": 1, "kind": "oracle",
+                         "sample": f"{curve} n={n_sample} per step, oracle.msm_pippenger s=8, 1 process"},
+        "e2e": {"value": val, "unit": "points/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+    return 0
+
+
+# ---------------------------------------------------------------------------------------
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--curve", default="bls12_381", choices=list(CURVE_INFO))
+    ap.add_argument("--log2n", type=int, default=26)
+    ap.add_argument("--window-bits", type=int, default=0)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--ref-sample", type=int, default=0)
+    ap.add_argument("--no-e2e", action="store_true")
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--check", action="store_true", help="verify the result against the oracle closed form")
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        return run_reference(args)
+
+    import numpy as np
+    import torch
+
+    import synth
+    from paper_conf_asplos_ji0x024_b200 import msm
+
+    ws, rank, local = dist_env()
+    assert ws == args.gpus, f"--gpus {args.gpus} but WORLD_SIZE {ws}"
+    torch.cuda.set_device(local)
+    dev = torch.device("cuda", local)
+    if ws > 1:
+        import torch.distributed as dist
+        dist.init_process_group("nccl", device_id=dev)
+    curve = args.curve
+    L32, S, lam, L, W = CURVE_INFO[curve]
+    r = synth.CURVE_ORDERS[curve]
+    n = 1 << args.log2n
+    off = n * rank // ws
+    n_g = n * (rank + 1) // ws - off
+    seed = 20240427 + 3
+    e0, delta = synth.point_seeds(r, seed)
+
+    # inputs: points generated on the device by the library's generator (not timed),
+    # scalars drawn on the host (numpy PCG64) and uploaded once for the HBM-resident runs.
+    t0 = time.time()
+    pts = torch.empty((n_g, 2 * L32), dtype=torch.int32, device=dev)
+    msm.gen_points(curve, synth.progression_offset(r, e0, delta, off), delta, n_g, pts)
+    ks_host = synth.scalars_range(r, off, n_g, seed)
+    ks_pinned = torch.from_numpy(ks_host.view(np.int32)).pin_memory()
+    ks_dev = ks_pinned.to(dev, non_blocking=False)
+    ctx = msm.Context(curve, pts, ngpus=1, n=n_g)
+    del pts
+    torch.cuda.empty_cache()
+    if args.window_bits:
+        ctx.set_option(msm.OPT_WINDOW_BITS, args.window_bits)
+    setup_s = time.time() - t0
+    stream = torch.cuda.ExternalStream(ctx.stream(0), device=dev)
+    pw = msm.partial_words(curve)
+    partial = torch.zeros(pw, dtype=torch.int32, device=dev)
+    gathered = torch.zeros((ws, pw), dtype=torch.int32, device=dev)
+
+    def step(scalars):
+        if ws == 1:
+            return ctx.run_words(scalars)
+        ctx.run_partial(scalars, partial)
+        torch.distributed.all_gather_into_tensor(gathered, partial)
+        if rank == 0:
+            return msm.finalize(curve, gathered, ws)
+        return None
+
+    def barrier():
+        torch.cuda.synchronize()
+        if ws > 1:
+            torch.distributed.barrier()
+        torch.cuda.synchronize()
+
+    for _ in range(args.warmup):
+        step(ks_dev)
+    barrier()
+    # timed: HBM-resident scalars
+    ev = [(torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)) for _ in range(args.steps)]
+    acc_ms, stage = [], []
+    sampler = ClockSampler(local)
+    with sampler:
+        barrier()
+        for i in range(args.steps):
+            ev[i][0].record(stream)
+            res = step(ks_dev)
+            ev[i][1].record(stream)
+            st = ctx.stats()
+            acc_ms.append(st["accumulate_ms"])
+            stage.append(st)
+        barrier()
+    times = [a.elapsed_time(b) for a, b in ev]
+    my_ms = sum(times) / len(times)
+    t_all = torch.tensor([my_ms], dtype=torch.float64, device=dev)
+    if ws > 1:
+        torch.distributed.all_reduce(t_all, op=torch.distributed.ReduceOp.MAX)
+    ms = float(t_all.item())
+
+    # e2e: host (pinned) scalars through the same C-ABI call, H2D inside the timed region
+    e2e = None
+    if not args.no_e2e:
+        for _ in range(1):
+            step(ks_pinned.numpy() if ws == 1 else ks_pinned)
+        barrier()
+        t0 = time.perf_counter()
+        e_ms = []
+        for i in range(max(2, min(args.steps, 5))):
+            s0 = time.perf_counter()
+            step(ks_pinned.numpy() if ws == 1 else ks_pinned)
+            if ws > 1:
+                barrier()
+            e_ms.append((time.perf_counter() - s0) * 1e3)
+        e_t = torch.tensor([sum(e_ms) / len(e_ms)], dtype=torch.float64, device=dev)
+        if ws > 1:
+            torch.distributed.all_reduce(e_t, op=torch.distributed.ReduceOp.MAX)
+        e2e_ms = float(e_t.item())
+        e2e = {"value": n / (e2e_ms / 1e3), "unit": "points/s", "ms_per_step": e2e_ms,
+               "h2d_bytes_per_step": n * S * 4, "d2h_bytes_per_step": 2 * L32 * 4,
+               "timing": "host wall clock around msm_run with pinned host scalars (max over ranks)"}
+
+    check = None
+    if args.check and rank == 0:
+        check = verify(curve, n, e0, delta, seed, ctx if ws == 1 else None, ks_dev, res, msm)
+
+    if rank != 0:
+        ctx.close()
+        if ws > 1:
+            torch.distributed.barrier()
+            torch.distributed.destroy_process_group()
+        return 0
+
+    # roofline of the dominant kernel (k_accumulate): algorithmic IMAD-pipe slots per launch
+    st = stage[-1]
+    nonempty = ctx.get_option(msm.OPT_NONEMPTY)
+    pacc = int(st["entries"]) - int(nonempty)
+    slots = pacc * 10 * imad_slots_per_mult(L)
+    acc_avg_ms = sum(acc_ms) / len(acc_ms)
+    pk = peaks()
+    sm_max = pk.get("sm_max_mhz", 1965.0)
+    peak_slots = 148 * 64 * sm_max * 1e6
+    achieved = slots / (acc_avg_ms / 1e3)
+    clocks = sampler.summary()
+    cpu = None
+    if not args.no_cpu_baseline and ws == 1:
+        cpu = cpu_baseline(curve)
+    paper = PAPER_MS.get((curve, args.log2n, ws))
+    line = {
+        "metric": METRIC,
+        "value": n / (ms / 1e3),
+        "unit": "points/s",
+        "n_gpus": ws,
+        "steps": args.steps,
+        "warmup": args.warmup,
+        "ms_per_step": ms,
+        "higher_is_better": True,
+        "scaling": "strong",
+        "vs_baseline": None,
+        "dtype": "u32 (exact modular integer arithmetic, radix-2^%d limbs)" % W,
+        "data": "synthetic: P_i = (e0 + i*delta) G generated on device, k_i uniform on [0, r) (numpy PCG64)",
+        "config": {"workload": f"{curve} G1 MSM n=2^{args.log2n} (BASELINE.json config C4)" if (curve, args.log2n) == ("bls12_381", 26)
+                   else f"{curve} G1 MSM n=2^{args.log2n}",
+                   "curve": curve, "n": n, "window_bits": st["window_bits"], "nwin": st["nwin"],
+                   "parallelism": f"point-sharded x{ws}" + (" + NCCL all-gather of partials" if ws > 1 else ""),
+                   "scalars": "device-resident (HBM) for value; pinned host for e2e",
+                   "l2": "inputs >> L2 (points %.1f GB + scalars %.1f GB per step); no flush needed" % (
+                       n * (2 * L + 2) * 4 / 1e9, n * S * 4 / 1e9)},
+        "stages_ms": {k: round(v, 3) for k, v in st.items() if k.endswith("_ms")},
+        "latency_ms": {"mean": ms, "min": min(times), "max": max(times)},
+        "roofline": {"kernel": "k_accumulate", "bound": "alu", "achieved": achieved / 1e12, "peak": peak_slots / 1e12,
+                     "unit": "T IMAD-pipe slots/s", "frac": achieved / peak_slots, "traffic": None,
+                     "work": f"{pacc} PACC x 10 field mults x {imad_slots_per_mult(L)} slots",
+                     "peak_basis": f"148 SM x 64 IMAD slots/clk x {sm_max} MHz (clocks.max.sm); IMAD.WIDE = 2 slots (measured)",
+                     "field_mults_per_s": pacc * 10 / (acc_avg_ms / 1e3)},
+        "clocks": clocks,
+        "gpu_launches": int(st["acc_launches"]) * args.steps + (args.steps if ws > 1 else 0),
+        "setup_s": round(setup_s, 2),
+    }
+    if paper:
+        line["paper_context"] = {"ms": paper, "hardware": f"{ws}x A100 80GB (DistMSM, PAPER.md Table 3)"}
+    if e2e:
+        line["e2e"] = e2e
+    if cpu:
+        line["cpu_baseline"] = cpu
+    if check is not None:
+        line["check"] = check
+    print(json.dumps(line), flush=True)
+    ctx.close()
+    if ws > 1:
+        torch.distributed.barrier()
+        torch.distributed.destroy_process_group()
+    return 0
+
+
+def verify(curve, n, e0, delta, seed, ctx, ks_dev, res, msm):
+    """Closed-form check (oracle): Q = (e0 * sum k_i + delta * sum i k_i mod r) G."""
+    import numpy as np
+    import synth
+    from oracle import ec, msm as omsm
+    from oracle.curves import CURVES
+    c = CURVES[curve]
+    ks = synth.scalars_range(c.r, 0, n, seed)
+    S = ks.shape[1]
+    sk, sik = 0, 0
+    idx = np.arange(n, dtype=np.uint64)
+    for w in range(S):
+        col = ks[:, w].astype(np.uint64)
+        sk += int(col.sum()) << (32 * w)
+        for h in range(2):  # 16-bit halves keep i * half < 2^42, chunk sums < 2^62
+            half = (col >> np.uint64(16 * h)) & np.uint64(0xFFFF)
+            tot = 0
+            for a in range(0, n, 1 << 20):
+                tot += int((idx[a:a + (1 << 20)] * half[a:a + (1 << 20)]).sum())
+            sik += tot << (32 * w + 16 * h)
+    want = ec.to_output(omsm.closed_form_arith(sk, sik, e0, delta, c))
+    got = res if isinstance(res, tuple) else msm.point_from_words(res, msm.field_words(curve))
+    return {"closed_form_match": got == want}
+
+
+if __name__ == "__main__":
+    sys.exit(main())

@@ -1,0 +1,166 @@
+/*
+ * msm.h — C ABI of the B200-native multi-scalar multiplication library (libmsm.so).
+ *
+ * Operation (§2.2): given fixed curve points P_i and per-call scalars k_i,
+ *     Q = sum_{i<n} k_i * P_i      in G1 of the selected curve,
+ * computed by Pippenger's bucket method (§2.3, :141-143) with signed c-bit
+ * windows, a per-window bucket counting sort (§3.2.1, Alg. 3), XYZZ bucket
+ * accumulation (Alg. 4, §3.2.2), bucket reduce and window combine,
+ * points sharded over GPUs with the partial results gathered and added.
+ *
+ * Encoding (all integers are arrays of little-endian 32-bit words):
+ *   base-field element   L32 = msm_field_words(curve) words, canonical (< p)
+ *   affine point         2*L32 words: x then y.  (0, 0) encodes the point at infinity O
+ *                        (it is on none of the four curves because b != 0)
+ *   scalar               S = msm_scalar_words(curve) words, canonical (< r)
+ *   result               2*L32 words, canonical affine; O -> (0, 0)
+ *   partial (XYZZ)       msm_partial_words(curve) words: the library's internal projective
+ *                        form (Montgomery radix-2^W limbs); only meaningful as input to
+ *                        msm_finalize of the same curve.
+ * Word counts: BN254 L32=8 S=8; BLS12-377 12/8; BLS12-381 12/8; MNT4-753 24/24.
+ *
+ * Pointers: a pointer argument documented "host or device" is classified with
+ * cudaPointerGetAttributes; device pointers must be 16-byte aligned.  The library never
+ * keeps a caller pointer past the call that receives it.
+ *
+ * Errors: every int-returning call returns MSM_OK (0) or a negative MSM_ERR_* code; no
+ * C++ exception or abort crosses the ABI.  Create returns NULL on failure and the code is
+ * available from msm_last_error() (thread-local).  After MSM_ERR_SCALAR or MSM_ERR_POINT
+ * the context stays usable; after MSM_ERR_CUDA it should be destroyed.
+ *
+ * Threading: one call at a time per context; distinct contexts are independent.
+ */
+#ifndef MSM_H
+#define MSM_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+typedef enum { MSM_BN254 = 0, MSM_BLS12_377 = 1, MSM_BLS12_381 = 2, MSM_MNT4_753 = 3 } msm_curve;
+
+enum {
+  MSM_OK = 0,
+  MSM_ERR_ARG = -1,           /* NULL pointer, bad size or option                       */
+  MSM_ERR_CURVE = -2,         /* unknown curve id                                       */
+  MSM_ERR_CUDA = -3,          /* CUDA runtime error                                     */
+  MSM_ERR_OOM = -4,           /* device allocation failed                               */
+  MSM_ERR_NCCL = -5,          /* reserved (collectives run in the caller's process group) */
+  MSM_ERR_POINT = -6,         /* an input point is not on the curve or not canonical    */
+  MSM_ERR_SCALAR = -7,        /* a scalar is >= r                                       */
+  MSM_ERR_UNIMPLEMENTED = -8,
+  MSM_ERR_NO_DEVICE = -9      /* no CUDA device / fewer devices than requested          */
+};
+
+/* Options for msm_set_option / msm_get_option. */
+enum {
+  MSM_OPT_WINDOW_BITS = 1,    /* c in [2, 24]; 0 = automatic (cost model). Reallocates scratch. */
+  MSM_OPT_ACC_THREADS = 2,    /* accumulation threads per device; 0 = automatic            */
+  MSM_OPT_SEG_LEN = 3,        /* buckets per bucket-reduce segment; 0 = automatic          */
+  MSM_OPT_NWIN = 101,         /* (get only) number of windows floor(lambda/c) + 1           */
+  MSM_OPT_NONEMPTY = 102      /* (get only) non-empty buckets of the last run on device 0   */
+};
+
+/* Per-stage device times of the last msm_run on device 0 (CUDA events), milliseconds. */
+typedef struct {
+  float h2d_ms;         /* scalar upload (0 for device-resident scalars)   */
+  float sort_ms;        /* a2+a3: digits, histogram, scan, scatter         */
+  float accumulate_ms;  /* a4: bucket accumulation (k_accumulate)          */
+  float fixup_ms;       /* a4: boundary partial fix-up (k_fixup)           */
+  float reduce_ms;      /* a5: bucket reduce                               */
+  float combine_ms;     /* a6: window combine                              */
+  float finalize_ms;    /* a7: gather + final add + normalisation          */
+  float total_ms;       /* whole msm_run on device 0                       */
+  int window_bits;      /* c used                                          */
+  int nwin;             /* windows                                         */
+  int acc_threads;      /* threads of k_accumulate                         */
+  int acc_launches;     /* kernels launched by the last run (all devices)  */
+  uint64_t entries;     /* sorted (bucket, point) entries = PACC + bucket starts, device 0 */
+} msm_stats;
+
+typedef struct msm_context msm_context;
+
+/* Sizes of the encodings above (negative MSM_ERR_CURVE for an unknown curve). */
+int msm_field_words(int curve);
+int msm_scalar_words(int curve);
+int msm_scalar_bits(int curve);    /* lambda = bit length of r (Table 1) */
+int msm_partial_words(int curve);
+
+/* Number of visible CUDA devices (0 when none). */
+int msm_device_count(void);
+
+/*
+ * Create a context holding n points sharded over devices 0..ngpus-1 in contiguous shards
+ * [floor(g*n/G), floor((g+1)*n/G)).  `points` (host or device, n*2*L32 words) is copied,
+ * converted to the device representation and checked on the curve; the caller keeps
+ * ownership.  n may be 0.  All scratch for msm_run is allocated here.
+ * Returns NULL on error (msm_last_error(): MSM_ERR_ARG/CURVE/NO_DEVICE/OOM/CUDA/POINT).
+ */
+msm_context* msm_context_create(int curve, const uint32_t* points, size_t n, int ngpus);
+
+/* NULL-safe; frees all device memory and streams of the context. */
+void msm_context_destroy(msm_context* ctx);
+
+/*
+ * Q = sum k_i P_i.  `scalars`: n*S words, host or device (device 0 for ngpus > 1 is
+ * copied peer-to-peer).  `result`: host buffer of 2*L32 words (written only on MSM_OK).
+ * Synchronous.  Returns MSM_OK, MSM_ERR_SCALAR (some k_i >= r), MSM_ERR_ARG, MSM_ERR_CUDA.
+ */
+int msm_run(msm_context* ctx, const uint32_t* scalars, uint32_t* result);
+
+/*
+ * The per-process half of a multi-process MSM (one process per GPU, ngpus == 1 contexts):
+ * computes this context's partial sum sum_{i in shard} k_i P_i and writes it in XYZZ form
+ * (msm_partial_words words) to `partial` (host or device).  Synchronous.
+ */
+int msm_run_partial(msm_context* ctx, const uint32_t* scalars, uint32_t* partial);
+
+/*
+ * Adds `count` XYZZ partials (host or device, count*msm_partial_words words) and writes
+ * the canonical affine result to the host buffer `result`.  Runs on the current device.
+ */
+int msm_finalize(int curve, const uint32_t* partials, int count, uint32_t* result);
+
+int msm_set_option(msm_context* ctx, int key, long value);
+long msm_get_option(msm_context* ctx, int key);
+int msm_get_stats(const msm_context* ctx, msm_stats* out);
+
+/* cudaStream_t of device `dev` of the context (as void*), for event timing by callers. */
+void* msm_get_stream(msm_context* ctx, int dev);
+
+int msm_last_error(void);
+const char* msm_error_string(int code);
+
+/*
+ * Synthetic input generator (not on the MSM path; used by bench.py and large tests):
+ * writes P_i = (e0 + i*delta) * G, i < n, as canonical affine words to `out` (device
+ * pointer, n*2*L32 words) on the current device.  e0, delta: S words each (host).
+ */
+int msm_gen_points(int curve, const uint32_t* e0, const uint32_t* delta, size_t n, uint32_t* out);
+
+/*
+ * Test-only entry points (host buffers; run on the current device; synchronous).
+ *   msm_debug_field: op 0 mul, 1 sqr, 2 add, 3 sub, 4 inv, 5 neg on n canonical
+ *     elements a[i], b[i] (L32 words each); out[i] canonical.
+ *   msm_debug_ec: op 0 acc (P + Q via Alg. 4 with P in XYZZ scaled by z1), 1 add (Alg. 1,
+ *     both scaled by z1/z2), 2 dbl; P, Q affine (2*L32 words, (0,0) = O); z: 2*L32 words
+ *     per element (z1, z2 non-zero canonical); out: affine.
+ *   msm_debug_digits: signed digits, out[i*nwin + j] (int32), nwin = floor(lambda/c)+1.
+ *   msm_debug_windows: runs msm_run's pipeline on the context (ngpus == 1) and writes the
+ *     window sums W_j (nwin affine points) to `windows`; if `buckets` is non-NULL also the
+ *     bucket sums B_{j,b} for b = 0..2^(c-1) (nwin*(2^(c-1)+1) affine points, O where empty).
+ */
+int msm_debug_field(int curve, int op, const uint32_t* a, const uint32_t* b, size_t n, uint32_t* out);
+int msm_debug_ec(int curve, int op, const uint32_t* P, const uint32_t* Q, const uint32_t* z, size_t n,
+                 uint32_t* out);
+int msm_debug_digits(int curve, int c, const uint32_t* scalars, size_t n, int32_t* out);
+int msm_debug_windows(msm_context* ctx, const uint32_t* scalars, uint32_t* windows, uint32_t* buckets);
+
+#ifdef __cplusplus
+}
+#endif
+
+#endif /* MSM_H */

@@ -1,0 +1,530 @@
+// Host runtime and C ABI of libmsm.so (include/msm.h).
+//
+// One context = n points sharded over G devices (contiguous shards).  Per
+// device the MSM pipeline of SURVEY.md §3.3 runs on the shard's own stream:
+//   H2D scalars -> k_digit_counts -> scan (3 kernels) -> k_digit_scatter      (a2, a3)
+//   -> k_accumulate -> k_fixup                                                (a4)
+//   -> k_bucket_segments -> k_sum_groups (x levels)                           (a5)
+//   -> k_window_combine                                                       (a6)
+// then the G partial XYZZ points meet on device 0 (peer copies) for k_finalize (a7).
+// For one-process-per-GPU jobs the caller gathers msm_run_partial() outputs itself
+// (torch.distributed / NCCL) and calls msm_finalize().
+#include <algorithm>
+#include <cmath>
+#include <cstring>
+#include <memory>
+#include <mutex>
+#include <new>
+#include <vector>
+
+#include "runtime.h"
+
+using namespace msmrt;
+
+static thread_local int g_last_error = MSM_OK;
+
+struct msm_context {
+  int curve = 0;
+  size_t n = 0;
+  int ngpus = 1;
+  std::vector<Shard> shards;
+  Options opt;
+  msm_stats stats{};
+  CurveOps* ops = nullptr;
+  int launches = 0;
+};
+
+namespace {
+
+bool is_device_ptr(const void* p, int* dev) {
+  cudaPointerAttributes a;
+  if (cudaPointerGetAttributes(&a, p) != cudaSuccess) {
+    cudaGetLastError();
+    return false;
+  }
+  if (a.type == cudaMemoryTypeDevice || a.type == cudaMemoryTypeManaged) {
+    if (dev) *dev = a.device;
+    return true;
+  }
+  return false;
+}
+
+// Pippenger cost model (field multiplications): per window n PACC (10 mults)
+// plus 2 PADD per bucket in the reduce (14 mults) over 2^(c-1) buckets.
+int choose_c(size_t n, int lambda) {
+  if (n == 0) return 8;
+  double best = 1e300;
+  int bc = 8;
+  for (int c = 4; c <= 22; c++) {
+    double cost = num_windows(lambda, c) * ((double)n * 10.0 + std::ldexp(1.0, c - 1) * 2 * 14.0);
+    if (cost < best) { best = cost; bc = c; }
+  }
+  return bc;
+}
+
+CurveOps* ops_for(int curve) {
+  switch (curve) {
+    case MSM_BN254: return make_ops_bn254();
+    case MSM_BLS12_377: return make_ops_bls12_377();
+    case MSM_BLS12_381: return make_ops_bls12_381();
+    case MSM_MNT4_753: return make_ops_mnt4_753();
+    default: return nullptr;
+  }
+}
+
+void destroy_shard(CurveOps* ops, Shard& s) {
+  cudaSetDevice(s.dev);
+  if (s.stream) cudaStreamSynchronize(s.stream);
+  if (ops) ops->free_scratch(s);
+  dfree(s.pts); dfree(s.scal); dfree(s.partial); dfree(s.partials); dfree(s.err); dfree(s.result);
+  if (s.host_err) cudaFreeHost(s.host_err);
+  s.host_err = nullptr;
+  for (auto& e : s.ev)
+    if (e) { cudaEventDestroy(e); e = nullptr; }
+  if (s.stream) cudaStreamDestroy(s.stream);
+  s.stream = nullptr;
+}
+
+int apply_window_bits(msm_context* ctx) {
+  for (auto& s : ctx->shards) {
+    int c = ctx->opt.c > 0 ? ctx->opt.c : choose_c(s.n, ctx->ops->lambda());
+    ctx->ops->configure(ctx->opt, s, c);
+  }
+  return MSM_OK;
+}
+
+// scalar pointer for shard s: device-resident on the shard's device -> use directly,
+// otherwise copy into s.scal (H2D or peer).
+const uint32_t* stage_scalars(msm_context* ctx, Shard& s, const uint32_t* scalars, bool is_dev, int src_dev) {
+  const size_t S = ctx->ops->S();
+  const uint32_t* src = scalars + s.off * S;
+  const size_t bytes = s.n * S * 4;
+  if (s.n == 0) return s.scal;
+  if (is_dev && src_dev == s.dev && ((uintptr_t)src % 16) == 0) return src;
+  if (is_dev) {
+    if (src_dev == s.dev) CK(cudaMemcpyAsync(s.scal, src, bytes, cudaMemcpyDeviceToDevice, s.stream));
+    else CK(cudaMemcpyPeerAsync(s.scal, s.dev, src, src_dev, bytes, s.stream));
+  } else {
+    CK(cudaMemcpyAsync(s.scal, src, bytes, cudaMemcpyHostToDevice, s.stream));
+  }
+  return s.scal;
+}
+
+int check_errors(msm_context* ctx) {
+  uint32_t e = 0;
+  for (auto& s : ctx->shards) {
+    CK(cudaSetDevice(s.dev));
+    CK(cudaMemcpyAsync(s.host_err, s.err, 4, cudaMemcpyDeviceToHost, s.stream));
+    CK(cudaStreamSynchronize(s.stream));
+    e |= *s.host_err;
+  }
+  if (e & 4u) return MSM_ERR_SCALAR;
+  if (e & 3u) return MSM_ERR_POINT;
+  return MSM_OK;
+}
+
+// runs a2..a6 on every shard; partials end in shard0.partials[g]
+int run_all(msm_context* ctx, const uint32_t* scalars, bool gather_to_dev0) {
+  int src_dev = -1;
+  const bool is_dev = ctx->n ? is_device_ptr(scalars, &src_dev) : false;
+  ctx->launches = 0;
+  const int XW = ctx->ops->XW();
+  Shard& s0 = ctx->shards[0];
+  for (size_t g = 0; g < ctx->shards.size(); g++) {
+    Shard& s = ctx->shards[g];
+    CK(cudaSetDevice(s.dev));
+    const bool timed = g == 0;
+    if (timed) CK(cudaEventRecord(s.ev[EV_START], s.stream));
+    CK(cudaMemsetAsync(s.err, 0, 4, s.stream));
+    const uint32_t* sc = stage_scalars(ctx, s, scalars, is_dev, src_dev);
+    ctx->launches += ctx->ops->enqueue_pipeline(s, sc, timed);
+  }
+  if (gather_to_dev0) {
+    for (size_t g = 0; g < ctx->shards.size(); g++) {
+      Shard& s = ctx->shards[g];
+      if (g == 0) {
+        CK(cudaSetDevice(s0.dev));
+        CK(cudaMemcpyAsync(s0.partials, s0.partial, XW * 4, cudaMemcpyDeviceToDevice, s0.stream));
+      } else {
+        CK(cudaSetDevice(s.dev));
+        CK(cudaEventRecord(s.ev[EV_END], s.stream));
+        CK(cudaSetDevice(s0.dev));
+        CK(cudaStreamWaitEvent(s0.stream, s.ev[EV_END], 0));
+        CK(cudaMemcpyPeerAsync(s0.partials + g * XW, s0.dev, s.partial, s.dev, XW * 4, s0.stream));
+      }
+    }
+  }
+  return MSM_OK;
+}
+
+void collect_stats(msm_context* ctx) {
+  Shard& s = ctx->shards[0];
+  CK(cudaSetDevice(s.dev));
+  CK(cudaEventSynchronize(s.ev[EV_END]));
+  auto el = [&](int a, int b) {
+    float ms = 0;
+    if (cudaEventElapsedTime(&ms, s.ev[a], s.ev[b]) != cudaSuccess) { cudaGetLastError(); ms = -1; }
+    return ms;
+  };
+  msm_stats& st = ctx->stats;
+  st.h2d_ms = el(EV_START, EV_H2D);
+  st.sort_ms = el(EV_H2D, EV_SORT);
+  st.accumulate_ms = el(EV_SORT, EV_ACC);
+  st.fixup_ms = el(EV_ACC, EV_FIX);
+  st.reduce_ms = el(EV_FIX, EV_RED);
+  st.combine_ms = el(EV_RED, EV_COMB);
+  st.finalize_ms = el(EV_COMB, EV_END);
+  st.total_ms = el(EV_START, EV_END);
+  st.window_bits = s.c;
+  st.nwin = s.nwin;
+  st.acc_threads = (int)s.acc_threads;
+  st.acc_launches = ctx->launches;
+  uint32_t M = 0;
+  cudaMemcpy(&M, s.goff + s.F, 4, cudaMemcpyDeviceToHost);
+  st.entries = M;
+}
+
+template <class F>
+int guarded(F&& f) {
+  try {
+    return f();
+  } catch (const CudaError& e) {
+    return e.code;
+  } catch (const std::bad_alloc&) {
+    return MSM_ERR_OOM;
+  } catch (...) {
+    return MSM_ERR_CUDA;
+  }
+}
+
+// small per-device scratch for msm_finalize (kept across calls; no cudaMalloc when timed)
+struct FinalizeScratch {
+  uint32_t* partials = nullptr;
+  size_t cap = 0;
+  uint32_t* result = nullptr;
+  cudaStream_t stream = nullptr;
+};
+std::mutex g_fin_mu;
+FinalizeScratch g_fin[64];
+
+}  // namespace
+
+// =========================================================================================
+extern "C" {
+
+int msm_field_words(int curve) {
+  CurveOps* o = ops_for(curve);
+  return o ? o->L32() : MSM_ERR_CURVE;
+}
+int msm_scalar_words(int curve) {
+  CurveOps* o = ops_for(curve);
+  return o ? o->S() : MSM_ERR_CURVE;
+}
+int msm_scalar_bits(int curve) {
+  CurveOps* o = ops_for(curve);
+  return o ? o->lambda() : MSM_ERR_CURVE;
+}
+int msm_partial_words(int curve) {
+  CurveOps* o = ops_for(curve);
+  return o ? o->XW() : MSM_ERR_CURVE;
+}
+
+int msm_device_count(void) {
+  int n = 0;
+  if (cudaGetDeviceCount(&n) != cudaSuccess) {
+    cudaGetLastError();
+    return 0;
+  }
+  return n;
+}
+
+int msm_last_error(void) { return g_last_error; }
+
+const char* msm_error_string(int code) {
+  switch (code) {
+    case MSM_OK: return "ok";
+    case MSM_ERR_ARG: return "invalid argument";
+    case MSM_ERR_CURVE: return "unknown curve";
+    case MSM_ERR_CUDA: return "CUDA error";
+    case MSM_ERR_OOM: return "device out of memory";
+    case MSM_ERR_NCCL: return "NCCL error";
+    case MSM_ERR_POINT: return "point not on curve or not canonical";
+    case MSM_ERR_SCALAR: return "scalar >= r";
+    case MSM_ERR_UNIMPLEMENTED: return "unimplemented";
+    case MSM_ERR_NO_DEVICE: return "no (or not enough) CUDA devices";
+    default: return "unknown error";
+  }
+}
+
+msm_context* msm_context_create(int curve, const uint32_t* points, size_t n, int ngpus) {
+  g_last_error = MSM_OK;
+  CurveOps* ops = ops_for(curve);
+  if (!ops) { g_last_error = MSM_ERR_CURVE; return nullptr; }
+  if (ngpus < 1 || (n > 0 && !points) || n >= 0x80000000ull) { g_last_error = MSM_ERR_ARG; return nullptr; }
+  const int ndev = msm_device_count();
+  if (ndev < 1 || ngpus > ndev) { g_last_error = MSM_ERR_NO_DEVICE; return nullptr; }
+  auto* ctx = new msm_context();
+  ctx->curve = curve;
+  ctx->n = n;
+  ctx->ngpus = ngpus;
+  ctx->ops = ops;
+  ctx->shards.resize(ngpus);
+  int rc = guarded([&]() -> int {
+    int src_dev = -1;
+    const bool in_dev = n ? is_device_ptr(points, &src_dev) : false;
+    const size_t pw_in = 2 * (size_t)ops->L32();
+    for (int g = 0; g < ngpus; g++) {
+      Shard& s = ctx->shards[g];
+      s.dev = g;
+      s.off = (size_t)((unsigned __int128)n * g / ngpus);
+      s.n = (size_t)((unsigned __int128)n * (g + 1) / ngpus) - s.off;
+      CK(cudaSetDevice(s.dev));
+      CK(cudaStreamCreateWithFlags(&s.stream, cudaStreamNonBlocking));
+      for (auto& e : s.ev) CK(cudaEventCreate(&e));
+      dalloc(&s.pts, s.n * ops->PW());
+      dalloc(&s.scal, s.n * ops->S());
+      dalloc(&s.partial, ops->XW());
+      dalloc(&s.err, 1);
+      dalloc(&s.result, 2 * ops->L32());
+      if (g == 0) dalloc(&s.partials, (size_t)ngpus * ops->XW());
+      CK(cudaMallocHost((void**)&s.host_err, 4));
+      CK(cudaMemsetAsync(s.err, 0, 4, s.stream));
+      if (s.n) {
+        const uint32_t* src = points + s.off * pw_in;
+        if (in_dev && src_dev == s.dev) {
+          ops->points_to_mont(s, src, s.n);
+        } else {
+          uint32_t* tmp;
+          dalloc(&tmp, s.n * pw_in);
+          if (in_dev) CK(cudaMemcpyPeerAsync(tmp, s.dev, src, src_dev, s.n * pw_in * 4, s.stream));
+          else CK(cudaMemcpyAsync(tmp, src, s.n * pw_in * 4, cudaMemcpyHostToDevice, s.stream));
+          ops->points_to_mont(s, tmp, s.n);
+          CK(cudaStreamSynchronize(s.stream));
+          dfree(tmp);
+        }
+      }
+    }
+    int e = check_errors(ctx);
+    if (e != MSM_OK) return e;
+    if (ngpus > 1) {
+      for (int a = 0; a < ngpus; a++)
+        for (int b = 0; b < ngpus; b++) {
+          if (a == b) continue;
+          int ok = 0;
+          cudaDeviceCanAccessPeer(&ok, a, b);
+          if (ok) {
+            cudaSetDevice(a);
+            cudaError_t pe = cudaDeviceEnablePeerAccess(b, 0);
+            if (pe != cudaSuccess) cudaGetLastError();
+          }
+        }
+    }
+    return apply_window_bits(ctx);
+  });
+  if (rc != MSM_OK) {
+    g_last_error = rc;
+    for (auto& s : ctx->shards) destroy_shard(ops, s);
+    delete ctx;
+    return nullptr;
+  }
+  return ctx;
+}
+
+void msm_context_destroy(msm_context* ctx) {
+  if (!ctx) return;
+  for (auto& s : ctx->shards) destroy_shard(ctx->ops, s);
+  delete ctx;
+}
+
+int msm_run(msm_context* ctx, const uint32_t* scalars, uint32_t* result) {
+  if (!ctx || !result || (ctx->n && !scalars)) return MSM_ERR_ARG;
+  return guarded([&]() -> int {
+    run_all(ctx, scalars, true);
+    Shard& s0 = ctx->shards[0];
+    CK(cudaSetDevice(s0.dev));
+    ctx->ops->enqueue_finalize(s0.partials, (int)ctx->shards.size(), s0.result, s0.stream);
+    ctx->launches++;
+    CK(cudaEventRecord(s0.ev[EV_END], s0.stream));
+    const int e = check_errors(ctx);
+    collect_stats(ctx);
+    if (e != MSM_OK) return e;
+    CK(cudaMemcpy(result, s0.result, 2 * ctx->ops->L32() * 4, cudaMemcpyDeviceToHost));
+    return MSM_OK;
+  });
+}
+
+int msm_run_partial(msm_context* ctx, const uint32_t* scalars, uint32_t* partial) {
+  if (!ctx || !partial || (ctx->n && !scalars) || ctx->shards.size() != 1) return MSM_ERR_ARG;
+  return guarded([&]() -> int {
+    run_all(ctx, scalars, false);
+    Shard& s0 = ctx->shards[0];
+    CK(cudaSetDevice(s0.dev));
+    CK(cudaEventRecord(s0.ev[EV_END], s0.stream));
+    const int e = check_errors(ctx);
+    collect_stats(ctx);
+    if (e != MSM_OK) return e;
+    int pdev = -1;
+    if (is_device_ptr(partial, &pdev)) {
+      if (pdev == s0.dev) CK(cudaMemcpyAsync(partial, s0.partial, ctx->ops->XW() * 4, cudaMemcpyDeviceToDevice, s0.stream));
+      else CK(cudaMemcpyPeerAsync(partial, pdev, s0.partial, s0.dev, ctx->ops->XW() * 4, s0.stream));
+      CK(cudaStreamSynchronize(s0.stream));
+    } else {
+      CK(cudaMemcpy(partial, s0.partial, ctx->ops->XW() * 4, cudaMemcpyDeviceToHost));
+    }
+    return MSM_OK;
+  });
+}
+
+int msm_finalize(int curve, const uint32_t* partials, int count, uint32_t* result) {
+  CurveOps* ops = ops_for(curve);
+  if (!ops) return MSM_ERR_CURVE;
+  if (count < 0 || (count > 0 && !partials) || !result) return MSM_ERR_ARG;
+  return guarded([&]() -> int {
+    int dev = 0;
+    CK(cudaGetDevice(&dev));
+    if (dev < 0 || dev >= 64) return MSM_ERR_ARG;
+    std::lock_guard<std::mutex> lk(g_fin_mu);
+    FinalizeScratch& fs = g_fin[dev];
+    const size_t words = (size_t)std::max(count, 1) * ops->XW();
+    if (!fs.stream) CK(cudaStreamCreateWithFlags(&fs.stream, cudaStreamNonBlocking));
+    if (fs.cap < words) {
+      dfree(fs.partials);
+      dalloc(&fs.partials, words);
+      fs.cap = words;
+    }
+    if (!fs.result) dalloc(&fs.result, 2 * 24);
+    const uint32_t* src = fs.partials;
+    int pdev = -1;
+    if (count > 0) {
+      if (is_device_ptr(partials, &pdev) && pdev == dev) src = partials;
+      else CK(cudaMemcpyAsync(fs.partials, partials, (size_t)count * ops->XW() * 4,
+                              pdev >= 0 ? cudaMemcpyDefault : cudaMemcpyHostToDevice, fs.stream));
+    }
+    ops->enqueue_finalize(src, count, fs.result, fs.stream);
+    CK(cudaMemcpyAsync(result, fs.result, 2 * ops->L32() * 4, cudaMemcpyDeviceToHost, fs.stream));
+    CK(cudaStreamSynchronize(fs.stream));
+    return MSM_OK;
+  });
+}
+
+int msm_set_option(msm_context* ctx, int key, long value) {
+  if (!ctx) return MSM_ERR_ARG;
+  switch (key) {
+    case MSM_OPT_WINDOW_BITS:
+      if (value != 0 && (value < 2 || value > 24)) return MSM_ERR_ARG;
+      ctx->opt.c = (int)value;
+      break;
+    case MSM_OPT_ACC_THREADS:
+      if (value < 0) return MSM_ERR_ARG;
+      ctx->opt.threads = (int)value;
+      break;
+    case MSM_OPT_SEG_LEN:
+      if (value < 0 || value > (1 << 20)) return MSM_ERR_ARG;
+      ctx->opt.seg = (int)value;
+      break;
+    default:
+      return MSM_ERR_ARG;
+  }
+  return guarded([&]() -> int { return apply_window_bits(ctx); });
+}
+
+long msm_get_option(msm_context* ctx, int key) {
+  if (!ctx) return MSM_ERR_ARG;
+  switch (key) {
+    case MSM_OPT_WINDOW_BITS: return ctx->shards[0].c;
+    case MSM_OPT_ACC_THREADS: return ctx->shards[0].acc_threads;
+    case MSM_OPT_SEG_LEN: return ctx->shards[0].seg;
+    case MSM_OPT_NWIN: return ctx->shards[0].nwin;
+    case MSM_OPT_NONEMPTY: {
+      long v = MSM_ERR_CUDA;
+      guarded([&]() -> int { CK(cudaSetDevice(ctx->shards[0].dev)); v = ctx->ops->count_nonempty(ctx->shards[0]); return MSM_OK; });
+      return v;
+    }
+    default: return MSM_ERR_ARG;
+  }
+}
+
+int msm_get_stats(const msm_context* ctx, msm_stats* out) {
+  if (!ctx || !out) return MSM_ERR_ARG;
+  *out = ctx->stats;
+  return MSM_OK;
+}
+
+void* msm_get_stream(msm_context* ctx, int dev) {
+  if (!ctx || dev < 0 || dev >= (int)ctx->shards.size()) return nullptr;
+  return (void*)ctx->shards[dev].stream;
+}
+
+int msm_gen_points(int curve, const uint32_t* e0, const uint32_t* delta, size_t n, uint32_t* out) {
+  CurveOps* ops = ops_for(curve);
+  if (!ops) return MSM_ERR_CURVE;
+  if (!e0 || !delta || (n && !out)) return MSM_ERR_ARG;
+  if (n && !is_device_ptr(out, nullptr)) return MSM_ERR_ARG;
+  return guarded([&]() -> int {
+    ops->gen_points(e0, delta, n, out);
+    return MSM_OK;
+  });
+}
+
+int msm_debug_field(int curve, int op, const uint32_t* a, const uint32_t* b, size_t n, uint32_t* out) {
+  CurveOps* ops = ops_for(curve);
+  if (!ops) return MSM_ERR_CURVE;
+  if (!a || !b || !out || op < 0 || op > 5) return MSM_ERR_ARG;
+  return guarded([&]() -> int {
+    ops->debug_field(op, a, b, n, out);
+    return MSM_OK;
+  });
+}
+
+int msm_debug_ec(int curve, int op, const uint32_t* P, const uint32_t* Q, const uint32_t* z, size_t n, uint32_t* out) {
+  CurveOps* ops = ops_for(curve);
+  if (!ops) return MSM_ERR_CURVE;
+  if (!P || !Q || !z || !out || op < 0 || op > 2) return MSM_ERR_ARG;
+  return guarded([&]() -> int {
+    ops->debug_ec(op, P, Q, z, n, out);
+    return MSM_OK;
+  });
+}
+
+int msm_debug_digits(int curve, int c, const uint32_t* scalars, size_t n, int32_t* out) {
+  CurveOps* ops = ops_for(curve);
+  if (!ops) return MSM_ERR_CURVE;
+  if (!scalars || !out || c < 2 || c > 30) return MSM_ERR_ARG;
+  return guarded([&]() -> int {
+    ops->debug_digits(c, scalars, n, out);
+    return MSM_OK;
+  });
+}
+
+int msm_debug_windows(msm_context* ctx, const uint32_t* scalars, uint32_t* windows, uint32_t* buckets) {
+  if (!ctx || !windows || (ctx->n && !scalars) || ctx->shards.size() != 1) return MSM_ERR_ARG;
+  return guarded([&]() -> int {
+    run_all(ctx, scalars, false);
+    Shard& s = ctx->shards[0];
+    CK(cudaSetDevice(s.dev));
+    CK(cudaEventRecord(s.ev[EV_END], s.stream));
+    int e = check_errors(ctx);
+    if (e != MSM_OK) return e;
+    const int L32 = ctx->ops->L32();
+    uint32_t* dout;
+    dalloc(&dout, (size_t)s.nwin * 2 * L32);
+    ctx->ops->to_affine(s.W, s.nwin, dout, s.stream);
+    CK(cudaMemcpyAsync(windows, dout, (size_t)s.nwin * 2 * L32 * 4, cudaMemcpyDeviceToHost, s.stream));
+    CK(cudaStreamSynchronize(s.stream));
+    dfree(dout);
+    if (buckets) {
+      std::vector<uint32_t> goff(s.F + 1);
+      CK(cudaMemcpy(goff.data(), s.goff, (s.F + 1) * 4, cudaMemcpyDeviceToHost));
+      dalloc(&dout, s.F * 2 * L32);
+      ctx->ops->to_affine(s.buckets, s.F, dout, s.stream);
+      CK(cudaMemcpyAsync(buckets, dout, s.F * 2 * L32 * 4, cudaMemcpyDeviceToHost, s.stream));
+      CK(cudaStreamSynchronize(s.stream));
+      dfree(dout);
+      for (size_t f = 0; f < s.F; f++)
+        if (goff[f + 1] == goff[f]) std::memset(buckets + f * 2 * L32, 0, 2 * L32 * 4);
+    }
+    return MSM_OK;
+  });
+}
+
+}  // extern "C"

@@ -1,0 +1,310 @@
+// Field layer: Montgomery arithmetic over F_p on radix-2^W limbs.
+//
+// What it computes is PAPER.md Alg. 2: C = A*B*R^-1 mod p with the
+// word-serial m[i] = C[i]*n'_0.  How it computes it is B200-specific
+// (DESIGN.md "Field layer"):
+//   * limbs are W = 30 (29 for MNT4-753) bits in 32-bit registers, R = 2^(W*L);
+//   * every limb product is one IMAD.WIDE.U32 (32x32 -> 64 with 64-bit addend), which
+//     runs at the full 64/clk/SM IMAD rate on sm_100a, whereas IMAD.HI.U32 runs at
+//     half rate (microbench/imad_peak.cu); a column of products accumulates in a 64-bit
+//     register with no carry propagation (finely-integrated product scanning, the FIPS
+//     variant PAPER.md:119 cites from [23]);
+//   * lazy reduction: values are kept in [0, B*p) with B <= KMAX and
+//     limbs normalised (< 2^W); a Montgomery product of inputs < 10p is < 2p
+//     (tools/gen_params.py asserts it per curve).  Only values leaving the library are
+//     fully reduced.
+#pragma once
+#include <cstdint>
+#include "params.h"
+
+typedef unsigned long long u64;
+
+#define DEVI __device__ __forceinline__
+
+// One IMAD.WIDE.U32 (a*b + c, 64-bit addend).  The product is an explicit PTX
+// mul.wide.u32 and the add is C++: ptxas then emits a clean IMAD.WIDE.U32 chain.
+// (An inline-asm mad.wide.u32 chain gets re-associated into IMAD.WIDE + IADD3 trees,
+// and a C++ (u64)a*b with a constant b becomes a 64x64 multiply with dead hi-word
+// adds — both checked with cuobjdump -sass.)
+DEVI u64 mad_wide(uint32_t a, uint32_t b, u64 c) {
+  u64 p;
+  asm("mul.wide.u32 %0, %1, %2;" : "=l"(p) : "r"(a), "r"(b));
+  return p + c;
+}
+
+template <class C>
+struct Fp {
+  static constexpr int L = C::L;
+  uint32_t v[C::L];
+};
+
+// ---- r = a*b*R^-1 mod p (lazy: result < 2p for inputs < 10p) ----
+template <class C>
+DEVI void fmul(uint32_t* r, const uint32_t* a, const uint32_t* b) {
+  constexpr int L = C::L, W = C::W;
+  constexpr uint32_t MASK = (1u << W) - 1;
+  uint32_t m[L];
+  if constexpr (C::NACC == 2) {
+    u64 cA = 0, cM = 0;
+#pragma unroll
+    for (int k = 0; k < 2 * L - 1; k++) {
+      const int lo = k - L + 1 > 0 ? k - L + 1 : 0;
+      const int hiA = k < L - 1 ? k : L - 1;
+      const int hiM = (k - 1) < (L - 1) ? k - 1 : L - 1;
+      u64 accA = cA, accM = cM;
+#pragma unroll
+      for (int i = lo; i <= hiA; i++) accA = mad_wide(a[i], b[k - i], accA);
+#pragma unroll
+      for (int i = lo; i <= hiM; i++) accM = mad_wide(m[i], C::P(k - i), accM);
+      if (k < L) {
+        uint32_t s = (uint32_t)accA + (uint32_t)accM;
+        m[k] = (s * C::N0) & MASK;
+        accM = mad_wide(m[k], C::P(0), accM);
+        uint32_t loA = (uint32_t)accA & MASK, loM = (uint32_t)accM & MASK;
+        cA = accA >> W;
+        cM = (accM >> W) + ((loA + loM) >> W);
+      } else {
+        uint32_t s = ((uint32_t)accA & MASK) + ((uint32_t)accM & MASK);
+        r[k - L] = s & MASK;
+        cA = accA >> W;
+        cM = (accM >> W) + (s >> W);
+      }
+    }
+    r[L - 1] = (uint32_t)(cA + cM);
+  } else {
+    u64 c = 0;
+#pragma unroll
+    for (int k = 0; k < 2 * L - 1; k++) {
+      const int lo = k - L + 1 > 0 ? k - L + 1 : 0;
+      const int hiA = k < L - 1 ? k : L - 1;
+      const int hiM = (k - 1) < (L - 1) ? k - 1 : L - 1;
+      u64 acc = c;
+#pragma unroll
+      for (int i = lo; i <= hiA; i++) acc = mad_wide(a[i], b[k - i], acc);
+#pragma unroll
+      for (int i = lo; i <= hiM; i++) acc = mad_wide(m[i], C::P(k - i), acc);
+      if (k < L) {
+        m[k] = ((uint32_t)acc * C::N0) & MASK;
+        acc = mad_wide(m[k], C::P(0), acc);
+      } else {
+        r[k - L] = (uint32_t)acc & MASK;
+      }
+      c = acc >> W;
+    }
+    r[L - 1] = (uint32_t)c;
+  }
+}
+
+// r = a^2 (same contract as fmul)
+template <class C>
+DEVI void fsqr(uint32_t* r, const uint32_t* a) { fmul<C>(r, a, a); }
+
+// r = a + b (no reduction; bound(r) = bound(a) + bound(b) <= KMAX)
+template <class C>
+DEVI void fadd(uint32_t* r, const uint32_t* a, const uint32_t* b) {
+  constexpr int L = C::L, W = C::W;
+  constexpr uint32_t MASK = (1u << W) - 1;
+  uint32_t c = 0;
+#pragma unroll
+  for (int i = 0; i < L - 1; i++) {
+    uint32_t s = a[i] + b[i] + c;
+    r[i] = s & MASK;
+    c = s >> W;
+  }
+  r[L - 1] = a[L - 1] + b[L - 1] + c;
+}
+
+// r = a - b + K*p   (requires bound(b) <= K; bound(r) = bound(a) + K)
+template <class C, int K>
+DEVI void fsub(uint32_t* r, const uint32_t* a, const uint32_t* b) {
+  static_assert(K < C::KMAX, "K*p not tabulated");
+  constexpr int L = C::L, W = C::W;
+  constexpr uint32_t MASK = (1u << W) - 1;
+  int32_t c = 0;
+#pragma unroll
+  for (int i = 0; i < L - 1; i++) {
+    int32_t s = (int32_t)(a[i] - b[i] + C::KP(K, i)) + c;
+    r[i] = (uint32_t)s & MASK;
+    c = s >> W;
+  }
+  r[L - 1] = (uint32_t)((int32_t)(a[L - 1] - b[L - 1] + C::KP(K, L - 1)) + c);
+}
+
+// r = K*p - a   (negation; requires bound(a) <= K)
+template <class C, int K>
+DEVI void fneg(uint32_t* r, const uint32_t* a) {
+  constexpr int L = C::L, W = C::W;
+  constexpr uint32_t MASK = (1u << W) - 1;
+  int32_t c = 0;
+#pragma unroll
+  for (int i = 0; i < L - 1; i++) {
+    int32_t s = (int32_t)(C::KP(K, i) - a[i]) + c;
+    r[i] = (uint32_t)s & MASK;
+    c = s >> W;
+  }
+  r[L - 1] = (uint32_t)((int32_t)(C::KP(K, L - 1) - a[L - 1]) + c);
+}
+
+template <class C>
+DEVI void fcopy(uint32_t* r, const uint32_t* a) {
+#pragma unroll
+  for (int i = 0; i < C::L; i++) r[i] = a[i];
+}
+
+template <class C>
+DEVI void fset_one(uint32_t* r) {
+#pragma unroll
+  for (int i = 0; i < C::L; i++) r[i] = C::ONE(i);
+}
+
+template <class C>
+DEVI void fzero(uint32_t* r) {
+#pragma unroll
+  for (int i = 0; i < C::L; i++) r[i] = 0;
+}
+
+// a == b as limb vectors (both normalised)
+template <class C>
+DEVI bool flimbs_eq(const uint32_t* a, const uint32_t* b) {
+  uint32_t d = 0;
+#pragma unroll
+  for (int i = 0; i < C::L; i++) d |= a[i] ^ b[i];
+  return d == 0;
+}
+
+// a == 0 (mod p) for a lazy value a < K*p.
+// a = j*p  <=>  a[0]*p^-1 = j (mod 2^W) and the limbs equal those of j*p.  The fast
+// reject costs one IMAD + one compare; the full compare runs only when j < K.
+template <class C, int K>
+DEVI bool fis_zero(const uint32_t* a) {
+  static_assert(K <= C::KMAX, "K*p not tabulated");
+  constexpr uint32_t MASK = (1u << C::W) - 1;
+  uint32_t j = (a[0] * C::PINV) & MASK;
+  if (j >= (uint32_t)K) return false;
+  uint32_t d = 0;
+#pragma unroll
+  for (int i = 0; i < C::L; i++) d |= a[i] ^ C::KPc()[j * C::L + i];
+  return d == 0;
+}
+
+// a == b (mod p) for lazy a, b < K*p
+template <class C, int K>
+DEVI bool fequal(const uint32_t* a, const uint32_t* b) {
+  uint32_t t[C::L];
+  fsub<C, K>(t, a, b);
+  return fis_zero<C, 2 * K>(t);
+}
+
+// conditional subtraction: if a >= k*p then a -= k*p (a normalised)
+template <class C, int k>
+DEVI void fcsub(uint32_t* a) {
+  constexpr int L = C::L, W = C::W;
+  constexpr uint32_t MASK = (1u << W) - 1;
+  uint32_t t[L];
+  int32_t c = 0;
+#pragma unroll
+  for (int i = 0; i < L; i++) {
+    int32_t s = (int32_t)(a[i] - C::KP(k, i)) + c;
+    t[i] = (uint32_t)s & MASK;
+    c = s >> W;
+  }
+  if (c >= 0) {
+#pragma unroll
+    for (int i = 0; i < L; i++) a[i] = t[i];
+  }
+}
+
+// full reduction to the canonical representative in [0, p), for a < 16p
+template <class C>
+DEVI void freduce(uint32_t* a) {
+  fcsub<C, 8>(a);
+  fcsub<C, 4>(a);
+  fcsub<C, 2>(a);
+  fcsub<C, 1>(a);
+}
+
+// radix-2^W limbs <-> 32-bit words (canonical values)
+template <class C>
+DEVI void from_words32(uint32_t* r, const uint32_t* w) {
+  constexpr int L = C::L, W = C::W;
+  constexpr uint32_t MASK = (1u << W) - 1;
+#pragma unroll
+  for (int i = 0; i < L; i++) {
+    const int bit = i * W, wi = bit >> 5, sh = bit & 31;
+    uint32_t lo = wi < C::L32 ? w[wi] : 0u;
+    uint32_t hi = (wi + 1) < C::L32 ? w[wi + 1] : 0u;
+    uint32_t v = sh ? ((lo >> sh) | (hi << (32 - sh))) : lo;
+    r[i] = v & MASK;
+  }
+}
+
+template <class C>
+DEVI void to_words32(uint32_t* w, const uint32_t* a) {
+  constexpr int L = C::L, W = C::W;
+#pragma unroll
+  for (int j = 0; j < C::L32; j++) {
+    uint32_t v = 0;
+#pragma unroll
+    for (int i = 0; i < L; i++) {
+      const int lo = i * W;  // limb i covers bits [lo, lo+W)
+      if (lo + W <= 32 * j || lo >= 32 * j + 32) continue;
+      const int sh = lo - 32 * j;
+      v |= sh >= 0 ? (a[i] << sh) : (a[i] >> (-sh));
+    }
+    w[j] = v;
+  }
+}
+
+// Montgomery form: x -> x*R mod p  (x canonical), and back (result canonical)
+template <class C>
+DEVI void fto_mont(uint32_t* r, const uint32_t* x) {
+  uint32_t r2[C::L];
+#pragma unroll
+  for (int i = 0; i < C::L; i++) r2[i] = C::R2(i);
+  fmul<C>(r, x, r2);
+}
+
+template <class C>
+DEVI void ffrom_mont(uint32_t* r, const uint32_t* a) {
+  uint32_t one[C::L];
+  one[0] = 1;
+#pragma unroll
+  for (int i = 1; i < C::L; i++) one[i] = 0;
+  fmul<C>(r, a, one);
+  freduce<C>(r);
+}
+
+template <class C>
+__device__ __noinline__ void fmul_ni(uint32_t* r, const uint32_t* a, const uint32_t* b) {
+  uint32_t x[C::L], y[C::L], z[C::L];
+  fcopy<C>(x, a);
+  fcopy<C>(y, b);
+  fmul<C>(z, x, y);
+  fcopy<C>(r, z);
+}
+
+// Multiplication as used by the EC layer: always inlined.  (An out-of-line copy for
+// MNT4-753 compiled faster, but sm_100a keeps the stack pointer in a uniform register, so
+// a warp whose lanes diverge between a path with a call and one touching the stack
+// corrupts local memory — compute-sanitizer caught it.  Rule in this code base: calls to
+// __noinline__ functions only from warp-uniform control flow.)
+template <class C>
+DEVI void fmul_e(uint32_t* r, const uint32_t* a, const uint32_t* b) { fmul<C>(r, a, b); }
+template <class C>
+DEVI void fsqr_e(uint32_t* r, const uint32_t* a) { fmul_e<C>(r, a, a); }
+
+// r = a^(p-2) = a^-1 (Montgomery form in and out; a != 0 mod p), Fermat (PAPER.md silent;
+// used only for the final affine normalisation)
+template <class C>
+__device__ __noinline__ void finv(uint32_t* r, const uint32_t* a) {
+  uint32_t acc[C::L];
+  fset_one<C>(acc);
+  for (int wi = C::L32 - 1; wi >= 0; wi--) {
+    const uint32_t e = C::PM2c()[wi];
+    for (int b = 31; b >= 0; b--) {
+      fmul_ni<C>(acc, acc, acc);
+      if ((e >> b) & 1u) fmul_ni<C>(acc, acc, a);
+    }
+  }
+  fcopy<C>(r, acc);
+}

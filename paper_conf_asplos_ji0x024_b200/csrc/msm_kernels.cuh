@@ -1,0 +1,673 @@
+// MSM kernels.  All templated on the curve parameter struct C.
+//
+// Data layout in HBM (per device shard):
+//   pts      [n][PW] u32      affine (x, y), Montgomery form, radix-2^W limbs, x then y,
+//                             padded to PW = round_up(2L, 4) words (16-B aligned records)
+//   scal     [n][S] u32       scalars k_i, canonical little-endian 32-bit words
+//   goff     [F+1] u32        F = nwin * NB flat buckets f = j*NB + b (NB = 2^(c-1) + 1);
+//                             exclusive prefix sum of the bucket counts over ALL windows
+//   cursor   [F] u32          scatter cursors (goff copy, consumed by atomics)
+//   sorted   [M] u32          point index | sign << 31, grouped by flat bucket
+//   buckets  [F] Xyzz         bucket sums B_{j,b} (valid where the bucket is non-empty)
+#pragma once
+#include "ec.cuh"
+
+namespace msmk {
+
+constexpr uint32_t SIGN_BIT = 0x80000000u;
+
+template <class C>
+struct Layout {
+  static constexpr int PW = ((2 * C::L + 3) / 4) * 4;  // words per stored affine point
+  static constexpr int XW = 4 * C::L;                   // words per XYZZ point
+};
+
+// ---------------------------------------------------------------------------------------
+// XYZZ load/store (plain word arrays; XYZZ records are 4L words)
+template <class C>
+DEVI void load_xyzz(Xyzz<C>& A, const uint32_t* __restrict__ p) {
+#pragma unroll
+  for (int i = 0; i < C::L; i++) {
+    A.X[i] = p[i];
+    A.Y[i] = p[C::L + i];
+    A.ZZ[i] = p[2 * C::L + i];
+    A.ZZZ[i] = p[3 * C::L + i];
+  }
+}
+template <class C>
+DEVI void store_xyzz(uint32_t* __restrict__ p, const Xyzz<C>& A) {
+#pragma unroll
+  for (int i = 0; i < C::L; i++) {
+    p[i] = A.X[i];
+    p[C::L + i] = A.Y[i];
+    p[2 * C::L + i] = A.ZZ[i];
+    p[3 * C::L + i] = A.ZZZ[i];
+  }
+}
+
+// gather one stored affine point with 16-B vector loads
+template <class C>
+DEVI void load_point(uint32_t* x, uint32_t* y, const uint32_t* __restrict__ pts, uint32_t idx) {
+  constexpr int PW = Layout<C>::PW;
+  uint32_t w[PW];
+  const uint4* src = reinterpret_cast<const uint4*>(pts + (size_t)idx * PW);
+#pragma unroll
+  for (int q = 0; q < PW / 4; q++) {
+    uint4 v = __ldg(src + q);
+    w[4 * q] = v.x; w[4 * q + 1] = v.y; w[4 * q + 2] = v.z; w[4 * q + 3] = v.w;
+  }
+#pragma unroll
+  for (int i = 0; i < C::L; i++) { x[i] = w[i]; y[i] = w[C::L + i]; }
+}
+
+// ---------------------------------------------------------------------------------------
+// a0: canonical affine words -> Montgomery radix-2^W, on-curve check (context creation)
+//     in: [n][2*L32] words, (0,0) = O.   err |= 1 for an off-curve point, 2 for x/y >= p.
+template <class C>
+__global__ void k_points_to_mont(uint32_t* __restrict__ pts, const uint32_t* __restrict__ in,
+                                 size_t n, uint32_t* err) {
+  constexpr int L = C::L, PW = Layout<C>::PW;
+  size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  uint32_t xw[C::L32], yw[C::L32];
+#pragma unroll
+  for (int k = 0; k < C::L32; k++) { xw[k] = in[i * 2 * C::L32 + k]; yw[k] = in[i * 2 * C::L32 + C::L32 + k]; }
+  uint32_t nz = 0;
+#pragma unroll
+  for (int k = 0; k < C::L32; k++) nz |= xw[k] | yw[k];
+  uint32_t x[L], y[L], out[PW];
+#pragma unroll
+  for (int k = 0; k < PW; k++) out[k] = 0;
+  if (nz) {
+    // range check x, y < p (canonical input)
+    bool ltx = false, lty = false, decx = false, decy = false;
+#pragma unroll
+    for (int k = C::L32 - 1; k >= 0; k--) {
+      const uint32_t pk = C::P32c()[k];
+      if (!decx && xw[k] != pk) { ltx = xw[k] < pk; decx = true; }
+      if (!decy && yw[k] != pk) { lty = yw[k] < pk; decy = true; }
+    }
+    if (!ltx || !lty) atomicOr(err, 2u);
+    from_words32<C>(x, xw);
+    from_words32<C>(y, yw);
+    fto_mont<C>(x, x);
+    fto_mont<C>(y, y);
+    // y^2 == x^3 + a x + b
+    uint32_t l[L], r[L], t[L], b[L];
+    fsqr_e<C>(l, y);
+    fsqr_e<C>(t, x);
+    fmul_e<C>(r, t, x);
+    if constexpr (!C::A_ZERO) {
+      uint32_t a[L];
+#pragma unroll
+      for (int k = 0; k < L; k++) a[k] = C::A_M(k);
+      fmul_e<C>(t, a, x);
+      fadd<C>(r, r, t);
+    }
+#pragma unroll
+    for (int k = 0; k < L; k++) b[k] = C::B_M(k);
+    fadd<C>(r, r, b);
+    if (!fequal<C, 6>(l, r)) atomicOr(err, 1u);
+#pragma unroll
+    for (int k = 0; k < L; k++) { out[k] = x[k]; out[L + k] = y[k]; }
+  }
+  uint4* dst = reinterpret_cast<uint4*>(pts + i * PW);
+#pragma unroll
+  for (int q = 0; q < PW / 4; q++) dst[q] = make_uint4(out[4 * q], out[4 * q + 1], out[4 * q + 2], out[4 * q + 3]);
+}
+
+// ---------------------------------------------------------------------------------------
+// a2: signed c-bit digits (R6):  nwin = floor(λ/c) + 1;  d_j = chunk_j + carry;
+//     for j < nwin-1: d_j > 2^(c-1) -> d_j -= 2^c, carry = 1.  Top digit never negated.
+template <class C>
+struct ScalarReg {
+  uint32_t w[C::S];
+};
+
+template <class C>
+DEVI void load_scalar(ScalarReg<C>& k, const uint32_t* __restrict__ scal, size_t i) {
+  if constexpr (C::S % 4 == 0) {
+    const uint4* src = reinterpret_cast<const uint4*>(scal + i * C::S);
+#pragma unroll
+    for (int q = 0; q < C::S / 4; q++) {
+      uint4 v = __ldg(src + q);
+      k.w[4 * q] = v.x; k.w[4 * q + 1] = v.y; k.w[4 * q + 2] = v.z; k.w[4 * q + 3] = v.w;
+    }
+  } else {
+#pragma unroll
+    for (int q = 0; q < C::S; q++) k.w[q] = scal[i * C::S + q];
+  }
+}
+
+// k < r ?
+template <class C>
+DEVI bool scalar_in_range(const ScalarReg<C>& k) {
+  bool lt = false, dec = false;
+#pragma unroll
+  for (int q = C::S - 1; q >= 0; q--) {
+    const uint32_t rq = C::R32c()[q];
+    if (!dec && k.w[q] != rq) { lt = k.w[q] < rq; dec = true; }
+  }
+  return lt;
+}
+
+// bits [bit, bit + c) of k, c <= 31
+template <class C>
+DEVI uint32_t scalar_bits(const ScalarReg<C>& k, int bit, int c) {
+  const int wi = bit >> 5, sh = bit & 31;
+  uint32_t lo = 0, hi = 0;
+#pragma unroll
+  for (int q = 0; q < C::S; q++) {
+    if (q == wi) lo = k.w[q];
+    if (q == wi + 1) hi = k.w[q];
+  }
+  uint64_t v = ((uint64_t)hi << 32) | lo;
+  return (uint32_t)(v >> sh) & ((1u << c) - 1u);
+}
+
+// Walks the windows of one scalar, calling f(j, bucket, negative) for non-zero digits.
+template <class C, class F>
+DEVI void for_each_digit(const ScalarReg<C>& k, int c, int nwin, F&& f) {
+  const uint32_t half = 1u << (c - 1);
+  uint32_t carry = 0;
+  for (int j = 0; j < nwin; j++) {
+    uint32_t d = scalar_bits<C>(k, j * c, c) + carry;
+    bool neg = false;
+    if (j < nwin - 1 && d > half) {
+      d = (1u << c) - d;
+      neg = true;
+      carry = 1;
+    } else {
+      carry = 0;
+    }
+    if (d) f(j, d, neg);
+  }
+}
+
+// histogram: counts[j*NB + b] += 1 for every non-zero digit.  err |= 4 for k >= r.
+template <class C>
+__global__ void k_digit_counts(const uint32_t* __restrict__ scal, size_t n, int c, int nwin,
+                               uint32_t NB, uint32_t* __restrict__ counts, uint32_t* err) {
+  size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  ScalarReg<C> k;
+  load_scalar<C>(k, scal, i);
+  if (!scalar_in_range<C>(k)) { atomicOr(err, 4u); return; }
+  for_each_digit<C>(k, c, nwin, [&](int j, uint32_t b, bool) { atomicAdd(counts + (size_t)j * NB + b, 1u); });
+}
+
+// scatter: sorted[cursor[f]++] = i | sign << 31
+template <class C>
+__global__ void k_digit_scatter(const uint32_t* __restrict__ scal, size_t n, int c, int nwin,
+                                uint32_t NB, uint32_t* __restrict__ cursor, uint32_t* __restrict__ sorted) {
+  size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  ScalarReg<C> k;
+  load_scalar<C>(k, scal, i);
+  if (!scalar_in_range<C>(k)) return;
+  for_each_digit<C>(k, c, nwin, [&](int j, uint32_t b, bool neg) {
+    uint32_t pos = atomicAdd(cursor + (size_t)j * NB + b, 1u);
+    sorted[pos] = (uint32_t)i | (neg ? SIGN_BIT : 0u);
+  });
+}
+
+// debug: digits[i][j] (signed int32)
+template <class C>
+__global__ void k_digits_debug(const uint32_t* __restrict__ scal, size_t n, int c, int nwin, int32_t* out) {
+  size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  ScalarReg<C> k;
+  load_scalar<C>(k, scal, i);
+  for (int j = 0; j < nwin; j++) out[i * nwin + j] = 0;
+  for_each_digit<C>(k, c, nwin, [&](int j, uint32_t b, bool neg) { out[i * nwin + j] = neg ? -(int32_t)b : (int32_t)b; });
+}
+
+// ---------------------------------------------------------------------------------------
+// exclusive scan of counts[0..F) -> goff[0..F], cursor[0..F)   (three-phase)
+constexpr int SCAN_THREADS = 1024;
+constexpr int SCAN_ITEMS = 8;
+constexpr int SCAN_TILE = SCAN_THREADS * SCAN_ITEMS;
+
+__device__ __forceinline__ uint32_t block_exclusive_scan(uint32_t v, uint32_t* smem, uint32_t* total) {
+  const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
+  uint32_t x = v;
+#pragma unroll
+  for (int o = 1; o < 32; o <<= 1) {
+    uint32_t y = __shfl_up_sync(0xffffffffu, x, o);
+    if (lane >= o) x += y;
+  }
+  if (lane == 31) smem[wid] = x;
+  __syncthreads();
+  if (wid == 0) {
+    uint32_t s = lane < (int)(blockDim.x >> 5) ? smem[lane] : 0u;
+#pragma unroll
+    for (int o = 1; o < 32; o <<= 1) {
+      uint32_t y = __shfl_up_sync(0xffffffffu, s, o);
+      if (lane >= o) s += y;
+    }
+    smem[lane] = s;
+  }
+  __syncthreads();
+  uint32_t warp_prefix = wid ? smem[wid - 1] : 0u;
+  if (total) *total = smem[(blockDim.x >> 5) - 1];
+  __syncthreads();
+  return warp_prefix + x - v;
+}
+
+static __global__ void k_scan_reduce(const uint32_t* __restrict__ counts, size_t F, uint32_t* __restrict__ tile_sums) {
+  __shared__ uint32_t smem[32];
+  size_t base = (size_t)blockIdx.x * SCAN_TILE + (size_t)threadIdx.x * SCAN_ITEMS;
+  uint32_t s = 0;
+#pragma unroll
+  for (int q = 0; q < SCAN_ITEMS; q++)
+    if (base + q < F) s += counts[base + q];
+  uint32_t tot;
+  block_exclusive_scan(s, smem, &tot);
+  if (threadIdx.x == 0) tile_sums[blockIdx.x] = tot;
+}
+
+// single block: exclusive scan of tile sums in place (ntiles arbitrary), writes total
+static __global__ void k_scan_tiles(uint32_t* tile_sums, size_t ntiles, uint32_t* total_out) {
+  __shared__ uint32_t smem[32];
+  uint32_t carry = 0;
+  for (size_t base = 0; base < ntiles; base += blockDim.x) {
+    size_t i = base + threadIdx.x;
+    uint32_t v = i < ntiles ? tile_sums[i] : 0u;
+    uint32_t tot;
+    uint32_t ex = block_exclusive_scan(v, smem, &tot);
+    if (i < ntiles) tile_sums[i] = carry + ex;
+    carry += tot;
+  }
+  if (threadIdx.x == 0) *total_out = carry;
+}
+
+static __global__ void k_scan_apply(const uint32_t* __restrict__ counts, size_t F, const uint32_t* __restrict__ tile_sums,
+                             uint32_t* __restrict__ goff, uint32_t* __restrict__ cursor) {
+  __shared__ uint32_t smem[32];
+  size_t base = (size_t)blockIdx.x * SCAN_TILE + (size_t)threadIdx.x * SCAN_ITEMS;
+  uint32_t v[SCAN_ITEMS];
+  uint32_t s = 0;
+#pragma unroll
+  for (int q = 0; q < SCAN_ITEMS; q++) {
+    v[q] = base + q < F ? counts[base + q] : 0u;
+    s += v[q];
+  }
+  uint32_t ex = block_exclusive_scan(s, smem, nullptr) + tile_sums[blockIdx.x];
+#pragma unroll
+  for (int q = 0; q < SCAN_ITEMS; q++) {
+    if (base + q < F) {
+      goff[base + q] = ex;
+      cursor[base + q] = ex;
+    }
+    ex += v[q];
+  }
+}
+
+// number of non-empty flat buckets (statistics only)
+static __global__ void k_count_nonempty(const uint32_t* __restrict__ goff, size_t F, unsigned long long* out) {
+  size_t f = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  unsigned v = (f < F && goff[f + 1] != goff[f]) ? 1u : 0u;
+  v = __reduce_add_sync(0xffffffffu, v);
+  if ((threadIdx.x & 31) == 0 && v) atomicAdd(out, (unsigned long long)v);
+}
+
+// ---------------------------------------------------------------------------------------
+// a4: bucket accumulation (PACC, Alg. 4), load-balanced over equal slices of `sorted`.
+//   Thread t owns entries [t*slice, min((t+1)*slice, M)).  Runs of equal flat bucket f are
+//   accumulated in registers.  A bucket whose first entry lies in the slice is written to
+//   buckets[f] (complete, or the owner's partial); a slice that starts inside a bucket
+//   writes its partial to carry[t] (carry_f[t] = f) for k_fixup.
+// Gathers the point of a sorted entry; negates y for a negative digit.  Returns false for
+// the point at infinity (stored as x = y = 0; y = 0 is on none of the curves since b != 0).
+template <class C>
+DEVI bool point_for_entry(uint32_t* x, uint32_t* y, const uint32_t* __restrict__ pts, uint32_t e) {
+  load_point<C>(x, y, pts, e & ~SIGN_BIT);
+  if (fis_zero<C, 2>(y)) return false;
+  if (e & SIGN_BIT) fneg<C, 2>(y, y);
+  return true;
+}
+
+template <class C>
+DEVI void acc_start(Xyzz<C>& acc, const uint32_t* x, const uint32_t* y, bool ok) {
+  if (ok) xyzz_from_affine<C>(acc, x, y);
+  else xyzz_set_zero<C>(acc);
+}
+
+// largest f with goff[f] <= e (goff non-decreasing, goff[0] = 0, e < goff[F])
+DEVI uint32_t find_bucket(const uint32_t* __restrict__ goff, uint32_t F, uint32_t e) {
+  uint32_t lo = 0, hi = F;  // invariant goff[lo] <= e < goff[hi]
+  while (hi - lo > 1) {
+    uint32_t mid = (lo + hi) >> 1;
+    if (__ldg(goff + mid) <= e) lo = mid; else hi = mid;
+  }
+  return lo;
+}
+
+template <class C>
+__global__ void __launch_bounds__(128) k_accumulate(const uint32_t* __restrict__ pts, const uint32_t* __restrict__ sorted,
+                                                    const uint32_t* __restrict__ goff, uint32_t F, uint32_t slice,
+                                                    uint32_t* __restrict__ buckets, uint32_t* __restrict__ carry_pts,
+                                                    int32_t* __restrict__ carry_f, uint32_t nthreads) {
+  constexpr int XW = Layout<C>::XW;
+  const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+  if (t >= nthreads) return;
+  const uint32_t M = __ldg(goff + F);
+  const uint64_t e0l = (uint64_t)t * slice;
+  if (e0l >= M) { carry_f[t] = -1; return; }
+  const uint32_t e0 = (uint32_t)e0l;
+  const uint32_t e1 = (uint32_t)(e0l + slice < (uint64_t)M ? e0l + slice : (uint64_t)M);
+  uint32_t f = find_bucket(goff, F, e0);
+  uint32_t end = __ldg(goff + f + 1);
+  bool head = __ldg(goff + f) < e0;
+  Xyzz<C> acc;
+  uint32_t x[C::L], y[C::L];
+  bool ok = point_for_entry<C>(x, y, pts, __ldg(sorted + e0));
+  acc_start<C>(acc, x, y, ok);
+  int32_t my_carry = -1;
+  for (uint32_t e = e0 + 1; e < e1; e++) {
+    const uint32_t ent = __ldg(sorted + e);
+    ok = point_for_entry<C>(x, y, pts, ent);
+    if (e == end) {
+      if (head) { store_xyzz<C>(carry_pts + (size_t)t * XW, acc); my_carry = (int32_t)f; head = false; }
+      else store_xyzz<C>(buckets + (size_t)f * XW, acc);
+      do { f++; end = __ldg(goff + f + 1); } while (end <= e);
+      acc_start<C>(acc, x, y, ok);
+    } else if (ok) {
+      xyzz_acc<C>(acc, x, y);
+    }
+  }
+  if (head) { store_xyzz<C>(carry_pts + (size_t)t * XW, acc); my_carry = (int32_t)f; }
+  else store_xyzz<C>(buckets + (size_t)f * XW, acc);
+  carry_f[t] = my_carry;
+}
+
+// Calls to __noinline__ EC functions below are made from warp-uniform control flow only
+// (loops with warp-uniform trip counts; per-lane differences become O operands): sm_100a
+// keeps the stack pointer in a uniform register, and lanes diverging around a call corrupt
+// local memory (found with compute-sanitizer).
+template <class C>
+DEVI void xyzz_select(Xyzz<C>& R, const Xyzz<C>& A, bool take) {
+  if (take) R = A;
+  else xyzz_set_zero<C>(R);
+}
+
+// run leaders sum the carries of their bucket and add them into buckets[f]
+template <class C>
+__global__ void k_fixup(uint32_t* __restrict__ buckets, const uint32_t* __restrict__ carry_pts,
+                        const int32_t* __restrict__ carry_f, uint32_t nthreads) {
+  constexpr int XW = Layout<C>::XW;
+  const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+  const int32_t f = t < nthreads ? carry_f[t] : -1;
+  const bool leader = f >= 0 && (t == 0 || carry_f[t - 1] != f);
+  const unsigned mask = __ballot_sync(0xffffffffu, leader);
+  if (!leader) return;
+  Xyzz<C> s, b;
+  load_xyzz<C>(s, carry_pts + (size_t)t * XW);
+  uint32_t u = t + 1;
+  bool more = u < nthreads && carry_f[u] == f;
+  while (__any_sync(mask, more)) {
+    if (more) load_xyzz<C>(b, carry_pts + (size_t)u * XW);
+    else xyzz_set_zero<C>(b);
+    __syncwarp(mask);
+    xyzz_add_ni<C>(s, s, b);
+    if (more) {
+      u++;
+      more = u < nthreads && carry_f[u] == f;
+    }
+  }
+  load_xyzz<C>(b, buckets + (size_t)f * XW);
+  __syncwarp(mask);
+  xyzz_add_ni<C>(s, s, b);
+  store_xyzz<C>(buckets + (size_t)f * XW, s);
+}
+
+// ---------------------------------------------------------------------------------------
+// a5: bucket reduce W_j = sum_{b=1}^{2^(c-1)} b * B_{j,b}.
+//   Segment t of window j covers buckets [lo, hi] = [1 + t*seg, min((t+1)*seg, 2^(c-1))]:
+//   descending running sum gives run = sum B_b and tri = sum (b - lo + 1) B_b;
+//   the segment's contribution is tri + (lo - 1) * run  (small-scalar double-and-add).
+// R = k * A by double-and-add over `bits` bits (warp-uniform trip count and call sequence)
+template <class C>
+DEVI void xyzz_mul_small(Xyzz<C>& R, const Xyzz<C>& A, uint32_t k, int bits) {
+  xyzz_set_zero<C>(R);
+  Xyzz<C> Z;
+  for (int b = bits - 1; b >= 0; b--) {
+    xyzz_dbl_ni<C>(R, R);
+    xyzz_select<C>(Z, A, (k >> b) & 1u);
+    xyzz_add_ni<C>(R, R, Z);
+  }
+}
+
+template <class C>
+__global__ void __launch_bounds__(128) k_bucket_segments(const uint32_t* __restrict__ buckets, const uint32_t* __restrict__ goff,
+                                                         int nwin, uint32_t NB, uint32_t seg, uint32_t nseg,
+                                                         uint32_t* __restrict__ out) {
+  constexpr int XW = Layout<C>::XW;
+  const uint32_t gid = blockIdx.x * blockDim.x + threadIdx.x;
+  if (gid >= (uint32_t)nwin * nseg) return;
+  const uint32_t j = gid / nseg, t = gid % nseg;
+  const uint32_t nb = NB - 1;  // buckets 1..nb
+  const uint32_t lo = 1 + t * seg;
+  Xyzz<C> run, tri, B;
+  xyzz_set_zero<C>(run);
+  xyzz_set_zero<C>(tri);
+  // uniform trip count `seg`; buckets past nb and empty buckets contribute O
+  for (uint32_t q = seg; q-- > 0;) {
+    const uint32_t b = lo + q;
+    const size_t f = (size_t)j * NB + b;
+    const bool ne = b <= nb && __ldg(goff + f + 1) != __ldg(goff + f);
+    if (ne) load_xyzz<C>(B, buckets + f * XW);
+    else xyzz_set_zero<C>(B);
+    xyzz_add_hot<C>(run, run, B);
+    xyzz_add_hot<C>(tri, tri, run);
+  }
+  int bits = 32 - __clz(nb);
+  xyzz_mul_small<C>(B, run, lo - 1, bits);
+  xyzz_add_ni<C>(tri, tri, B);
+  store_xyzz<C>(out + (size_t)gid * XW, tri);
+}
+
+// out[j*nout + g] = sum of in[j*nin + g*group .. + group)   (per window)
+template <class C>
+__global__ void __launch_bounds__(128) k_sum_groups(const uint32_t* __restrict__ in, uint32_t nin, uint32_t group,
+                                                    uint32_t nout, int nwin, uint32_t* __restrict__ out) {
+  constexpr int XW = Layout<C>::XW;
+  const uint32_t gid = blockIdx.x * blockDim.x + threadIdx.x;
+  if (gid >= (uint32_t)nwin * nout) return;
+  const uint32_t j = gid / nout, g = gid % nout;
+  Xyzz<C> s, b;
+  xyzz_set_zero<C>(s);
+  for (uint32_t q = 0; q < group; q++) {
+    const uint32_t i = g * group + q;
+    if (i < nin) load_xyzz<C>(b, in + ((size_t)j * nin + i) * XW);
+    else xyzz_set_zero<C>(b);
+    xyzz_add_ni<C>(s, s, b);
+  }
+  store_xyzz<C>(out + (size_t)gid * XW, s);
+}
+
+// ---------------------------------------------------------------------------------------
+// a6: window combine Q = sum_j 2^(j c) W_j (Horner), one thread.  Writes the XYZZ partial.
+template <class C>
+__global__ void k_window_combine(const uint32_t* __restrict__ W, int nwin, int c, uint32_t* __restrict__ partial) {
+  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  constexpr int XW = Layout<C>::XW;
+  Xyzz<C> Q, B;
+  load_xyzz<C>(Q, W + (size_t)(nwin - 1) * XW);
+  for (int j = nwin - 2; j >= 0; j--) {
+    for (int s = 0; s < c; s++) xyzz_dbl_ni<C>(Q, Q);
+    load_xyzz<C>(B, W + (size_t)j * XW);
+    xyzz_add_ni<C>(Q, Q, B);
+  }
+  store_xyzz<C>(partial, Q);
+}
+
+// a7: sum G partial XYZZ points, normalise to canonical affine 32-bit words
+template <class C>
+__global__ void k_finalize(const uint32_t* __restrict__ partials, int count, uint32_t* __restrict__ result) {
+  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  constexpr int XW = Layout<C>::XW;
+  Xyzz<C> Q, B;
+  xyzz_set_zero<C>(Q);
+  for (int g = 0; g < count; g++) {
+    load_xyzz<C>(B, partials + (size_t)g * XW);
+    xyzz_add_ni<C>(Q, Q, B);
+  }
+  xyzz_to_affine_words<C>(result, result + C::L32, Q);
+}
+
+// normalise an array of XYZZ points to affine words (debug: bucket / window sums)
+template <class C>
+__global__ void k_to_affine(const uint32_t* __restrict__ in, size_t n, uint32_t* __restrict__ out) {
+  size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  constexpr int XW = Layout<C>::XW;
+  Xyzz<C> A;
+  load_xyzz<C>(A, in + i * XW);
+  xyzz_to_affine_words<C>(out + i * 2 * C::L32, out + i * 2 * C::L32 + C::L32, A);
+}
+
+// ---------------------------------------------------------------------------------------
+// Synthetic point generator (bench / large tests; not on the MSM path):
+//   P_i = (e0 + i*delta) G = E0 + i*D, with E0 = e0 G, D = delta G computed by one thread.
+template <class C>
+DEVI void xyzz_mul_words(Xyzz<C>& R, const Xyzz<C>& A, const uint32_t* k, int nwords) {
+  xyzz_set_zero<C>(R);
+  Xyzz<C> Z;
+  for (int w = nwords - 1; w >= 0; w--) {
+    for (int b = 31; b >= 0; b--) {
+      xyzz_dbl_ni<C>(R, R);
+      xyzz_select<C>(Z, A, (k[w] >> b) & 1u);
+      xyzz_add_ni<C>(R, R, Z);
+    }
+  }
+}
+
+// base: G in canonical affine words; e0w / dw: S words each.  out2: [2] XYZZ (E0, D)
+template <class C>
+__global__ void k_gen_bases(const uint32_t* __restrict__ gw, const uint32_t* __restrict__ e0w,
+                            const uint32_t* __restrict__ dw, uint32_t* __restrict__ out2) {
+  if (threadIdx.x != 0 || blockIdx.x != 0) return;
+  constexpr int XW = Layout<C>::XW;
+  uint32_t x[C::L], y[C::L];
+  from_words32<C>(x, gw);
+  from_words32<C>(y, gw + C::L32);
+  fto_mont<C>(x, x);
+  fto_mont<C>(y, y);
+  Xyzz<C> G, R;
+  xyzz_from_affine<C>(G, x, y);
+  uint32_t k[C::S];
+  for (int q = 0; q < C::S; q++) k[q] = e0w[q];
+  xyzz_mul_words<C>(R, G, k, C::S);
+  store_xyzz<C>(out2, R);
+  for (int q = 0; q < C::S; q++) k[q] = dw[q];
+  xyzz_mul_words<C>(R, G, k, C::S);
+  store_xyzz<C>(out2 + XW, R);
+}
+
+// thread t generates points [t*chunk, min((t+1)*chunk, n)) as canonical affine words
+template <class C>
+__global__ void __launch_bounds__(128) k_gen_points(const uint32_t* __restrict__ bases, size_t n, uint32_t chunk,
+                                                    uint32_t* __restrict__ out) {
+  constexpr int XW = Layout<C>::XW;
+  const size_t t = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const size_t i0 = t * chunk;
+  if (i0 >= n) return;
+  Xyzz<C> E0, D, P, T;
+  load_xyzz<C>(E0, bases);
+  load_xyzz<C>(D, bases + XW);
+  uint32_t kw[2] = {(uint32_t)i0, (uint32_t)(i0 >> 32)};
+  xyzz_mul_words<C>(T, D, kw, 2);
+  xyzz_add_ni<C>(P, E0, T);
+  uint32_t w[2 * C::L32];
+  for (uint32_t q = 0; q < chunk; q++) {  // uniform trip count; tail lanes compute and drop
+    const size_t i = i0 + q;
+    xyzz_to_affine_words<C>(w, w + C::L32, P);
+    if (i < n)
+      for (int k = 0; k < 2 * C::L32; k++) out[i * 2 * C::L32 + k] = w[k];
+    xyzz_add_ni<C>(P, P, D);
+  }
+}
+
+// ---------------------------------------------------------------------------------------
+// debug kernels for the field / EC layers (tests only)
+enum { DBG_MUL = 0, DBG_SQR = 1, DBG_ADD = 2, DBG_SUB = 3, DBG_INV = 4, DBG_NEG = 5 };
+
+template <class C>
+__global__ void k_debug_field(int op, const uint32_t* __restrict__ a, const uint32_t* __restrict__ b, size_t n,
+                              uint32_t* __restrict__ out) {
+  size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  constexpr int L = C::L;
+  uint32_t x[L], y[L], r[L];
+  from_words32<C>(x, a + i * C::L32);
+  from_words32<C>(y, b + i * C::L32);
+  fto_mont<C>(x, x);
+  fto_mont<C>(y, y);
+  switch (op) {
+    case DBG_MUL: fmul_e<C>(r, x, y); break;
+    case DBG_SQR: fsqr_e<C>(r, x); break;
+    case DBG_ADD: fadd<C>(r, x, y); break;
+    case DBG_SUB: fsub<C, 2>(r, x, y); break;
+    case DBG_INV: finv<C>(r, x); break;
+    default: fneg<C, 2>(r, x); break;
+  }
+  ffrom_mont<C>(r, r);
+  to_words32<C>(out + i * C::L32, r);
+}
+
+enum { DBG_EC_ACC = 0, DBG_EC_ADD = 1, DBG_EC_DBL = 2 };
+
+// P, Q affine canonical words (2*L32), (0,0) = O; z1, z2 non-zero scalars (L32 words) used to
+// randomise the XYZZ representatives: (x z^2, y z^3, z^2, z^3).
+template <class C>
+DEVI void debug_xyzz_in(Xyzz<C>& A, const uint32_t* P, const uint32_t* zw) {
+  constexpr int L = C::L;
+  uint32_t x[L], y[L], z[L], z2[L], z3[L];
+  from_words32<C>(x, P);
+  from_words32<C>(y, P + C::L32);
+  uint32_t nz = 0;
+  for (int k = 0; k < 2 * C::L32; k++) nz |= P[k];
+  if (!nz) { xyzz_set_zero<C>(A); return; }
+  from_words32<C>(z, zw);
+  fto_mont<C>(x, x);
+  fto_mont<C>(y, y);
+  fto_mont<C>(z, z);
+  fsqr_e<C>(z2, z);
+  fmul_e<C>(z3, z2, z);
+  fmul_e<C>(A.X, x, z2);
+  fmul_e<C>(A.Y, y, z3);
+  fcopy<C>(A.ZZ, z2);
+  fcopy<C>(A.ZZZ, z3);
+}
+
+template <class C>
+__global__ void k_debug_ec(int op, const uint32_t* __restrict__ P, const uint32_t* __restrict__ Q,
+                           const uint32_t* __restrict__ z, size_t n, uint32_t* __restrict__ out) {
+  size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  constexpr int L = C::L;
+  const uint32_t* p = P + i * 2 * C::L32;
+  const uint32_t* q = Q + i * 2 * C::L32;
+  Xyzz<C> A, B, R;
+  debug_xyzz_in<C>(A, p, z + i * 2 * C::L32);
+  if (op == DBG_EC_ACC) {
+    uint32_t x[L], y[L];
+    from_words32<C>(x, q);
+    from_words32<C>(y, q + C::L32);
+    fto_mont<C>(x, x);
+    fto_mont<C>(y, y);
+    R = A;
+    uint32_t nz = 0;
+    for (int k = 0; k < 2 * C::L32; k++) nz |= q[k];
+    if (nz) xyzz_acc_ni<C>(R, x, y);
+  } else if (op == DBG_EC_ADD) {
+    debug_xyzz_in<C>(B, q, z + i * 2 * C::L32 + C::L32);
+    xyzz_add_ni<C>(R, A, B);
+  } else {
+    xyzz_dbl_ni<C>(R, A);
+  }
+  xyzz_to_affine_words<C>(out + i * 2 * C::L32, out + i * 2 * C::L32 + C::L32, R);
+}
+
+}  // namespace msmk

@@ -1,0 +1,224 @@
+// Per-curve implementation of msmrt::CurveOps: launches the kernels of msm_kernels.cuh.
+// Included by exactly one translation unit per curve (curve_*.cu).
+#pragma once
+#include <algorithm>
+#include <cmath>
+
+#include "msm_kernels.cuh"
+#include "runtime.h"
+
+namespace msmrt {
+
+using namespace msmk;
+
+template <class C>
+struct Ops final : CurveOps {
+  static constexpr int XW_ = Layout<C>::XW;
+  static constexpr int PW_ = Layout<C>::PW;
+  int L32() const override { return C::L32; }
+  int S() const override { return C::S; }
+  int lambda() const override { return C::LAMBDA; }
+  int PW() const override { return PW_; }
+  int XW() const override { return XW_; }
+
+  void points_to_mont(Shard& s, const uint32_t* in_dev, size_t n) override {
+    if (n == 0) return;
+    k_points_to_mont<C><<<(unsigned)cdiv(n, 128), 128, 0, s.stream>>>(s.pts, in_dev, n, s.err);
+    CK(cudaGetLastError());
+  }
+
+  void free_scratch(Shard& s) override {
+    dfree(s.counts); dfree(s.goff); dfree(s.cursor); dfree(s.sorted); dfree(s.buckets);
+    dfree(s.carry_pts); dfree(s.carry_f); dfree(s.segA); dfree(s.segB); dfree(s.W); dfree(s.tiles);
+  }
+
+  void configure(const Options& o, Shard& s, int c) override {
+    CK(cudaSetDevice(s.dev));
+    free_scratch(s);
+    s.c = c;
+    s.nwin = num_windows(C::LAMBDA, c);
+    s.NB = (1u << (c - 1)) + 1;
+    s.F = (size_t)s.nwin * s.NB;
+    s.ntiles = cdiv(s.F, SCAN_TILE);
+    cudaDeviceProp prop;
+    CK(cudaGetDeviceProperties(&prop, s.dev));
+    const int sms = prop.multiProcessorCount;
+    int bps = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_accumulate<C>, 128, 0));
+    if (bps < 1) bps = 1;
+    const size_t resident = (size_t)sms * bps * 128;
+    const size_t Mmax = s.n * (size_t)s.nwin;
+    size_t T = o.threads > 0 ? (size_t)o.threads : std::min(resident, std::max<size_t>(1, cdiv(Mmax, 16)));
+    if (T < 1) T = 1;
+    s.slice = (uint32_t)std::max<size_t>(1, cdiv(Mmax, T));
+    s.acc_threads = (uint32_t)std::max<size_t>(1, cdiv(Mmax, s.slice));
+    // bucket-reduce segments
+    int bps2 = 0;
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps2, k_bucket_segments<C>, 128, 0));
+    if (bps2 < 1) bps2 = 1;
+    const size_t resident2 = (size_t)sms * bps2 * 128;
+    const size_t nb = s.NB - 1;
+    uint32_t seg = o.seg > 0 ? (uint32_t)o.seg : 4;
+    if (o.seg <= 0)
+      while (seg < 4096 && (size_t)s.nwin * cdiv(nb, seg) > resident2) seg *= 2;
+    s.seg = seg;
+    s.nseg = (uint32_t)cdiv(nb, seg);
+    dalloc(&s.counts, s.F);
+    dalloc(&s.goff, s.F + 1);
+    dalloc(&s.cursor, s.F);
+    dalloc(&s.sorted, Mmax);
+    dalloc(&s.buckets, s.F * XW_);
+    dalloc(&s.carry_pts, (size_t)s.acc_threads * XW_);
+    dalloc(&s.carry_f, s.acc_threads);
+    dalloc(&s.segA, (size_t)s.nwin * s.nseg * XW_);
+    dalloc(&s.segB, (size_t)s.nwin * cdiv(s.nseg, 32) * XW_);
+    dalloc(&s.W, (size_t)s.nwin * XW_);
+    dalloc(&s.tiles, s.ntiles + 1);
+  }
+
+  int enqueue_pipeline(Shard& s, const uint32_t* scal, bool timed) override {
+    cudaStream_t st = s.stream;
+    int launches = 0;
+    const size_t n = s.n;
+    if (timed) CK(cudaEventRecord(s.ev[EV_H2D], st));
+    // a2 + a3: digits, histogram, scan, scatter
+    CK(cudaMemsetAsync(s.counts, 0, s.F * sizeof(uint32_t), st));
+    if (n) {
+      k_digit_counts<C><<<(unsigned)cdiv(n, 256), 256, 0, st>>>(scal, n, s.c, s.nwin, s.NB, s.counts, s.err);
+      launches++;
+    }
+    k_scan_reduce<<<(unsigned)s.ntiles, SCAN_THREADS, 0, st>>>(s.counts, s.F, s.tiles);
+    k_scan_tiles<<<1, 1024, 0, st>>>(s.tiles, s.ntiles, s.goff + s.F);
+    k_scan_apply<<<(unsigned)s.ntiles, SCAN_THREADS, 0, st>>>(s.counts, s.F, s.tiles, s.goff, s.cursor);
+    launches += 3;
+    if (n) {
+      k_digit_scatter<C><<<(unsigned)cdiv(n, 256), 256, 0, st>>>(scal, n, s.c, s.nwin, s.NB, s.cursor, s.sorted);
+      launches++;
+    }
+    CK(cudaGetLastError());
+    if (timed) CK(cudaEventRecord(s.ev[EV_SORT], st));
+    // a4: accumulate + fixup
+    k_accumulate<C><<<(unsigned)cdiv(s.acc_threads, 128), 128, 0, st>>>(s.pts, s.sorted, s.goff, (uint32_t)s.F, s.slice,
+                                                                        s.buckets, s.carry_pts, s.carry_f, s.acc_threads);
+    launches++;
+    CK(cudaGetLastError());
+    if (timed) CK(cudaEventRecord(s.ev[EV_ACC], st));
+    k_fixup<C><<<(unsigned)cdiv(s.acc_threads, 128), 128, 0, st>>>(s.buckets, s.carry_pts, s.carry_f, s.acc_threads);
+    launches++;
+    CK(cudaGetLastError());
+    if (timed) CK(cudaEventRecord(s.ev[EV_FIX], st));
+    // a5: bucket reduce
+    const uint32_t total = (uint32_t)s.nwin * s.nseg;
+    k_bucket_segments<C><<<(unsigned)cdiv(total, 128), 128, 0, st>>>(s.buckets, s.goff, s.nwin, s.NB, s.seg, s.nseg, s.segA);
+    launches++;
+    uint32_t nin = s.nseg;
+    uint32_t* src = s.segA;
+    uint32_t* dst = s.segB;
+    while (nin > 1) {
+      const uint32_t group = nin > 32 ? 32 : nin;
+      const uint32_t nout = (uint32_t)cdiv(nin, group);
+      uint32_t* out = nout == 1 ? s.W : dst;
+      k_sum_groups<C><<<(unsigned)cdiv((size_t)s.nwin * nout, 128), 128, 0, st>>>(src, nin, group, nout, s.nwin, out);
+      launches++;
+      nin = nout;
+      std::swap(src, dst);
+      if (nout == 1) { src = s.W; break; }
+    }
+    if (src != s.W) CK(cudaMemcpyAsync(s.W, src, (size_t)s.nwin * XW_ * 4, cudaMemcpyDeviceToDevice, st));
+    CK(cudaGetLastError());
+    if (timed) CK(cudaEventRecord(s.ev[EV_RED], st));
+    // a6: window combine
+    k_window_combine<C><<<1, 32, 0, st>>>(s.W, s.nwin, s.c, s.partial);
+    launches++;
+    CK(cudaGetLastError());
+    if (timed) CK(cudaEventRecord(s.ev[EV_COMB], st));
+    return launches;
+  }
+
+  void enqueue_finalize(const uint32_t* partials, int count, uint32_t* result, cudaStream_t st) override {
+    k_finalize<C><<<1, 32, 0, st>>>(partials, count, result);
+    CK(cudaGetLastError());
+  }
+
+  void gen_points(const uint32_t* e0, const uint32_t* delta, size_t n, uint32_t* out) override {
+    uint32_t *g, *e, *d, *bases;
+    dalloc(&g, 2 * C::L32);
+    dalloc(&e, C::S);
+    dalloc(&d, C::S);
+    dalloc(&bases, 2 * XW_);
+    try {
+      CK(cudaMemcpy(g, C::G_h, 2 * C::L32 * 4, cudaMemcpyHostToDevice));
+      CK(cudaMemcpy(e, e0, C::S * 4, cudaMemcpyHostToDevice));
+      CK(cudaMemcpy(d, delta, C::S * 4, cudaMemcpyHostToDevice));
+      k_gen_bases<C><<<1, 32>>>(g, e, d, bases);
+      CK(cudaGetLastError());
+      const uint32_t chunk = 64;
+      const size_t threads = cdiv(n, chunk);
+      if (threads) k_gen_points<C><<<(unsigned)cdiv(threads, 128), 128>>>(bases, n, chunk, out);
+      CK(cudaGetLastError());
+      CK(cudaDeviceSynchronize());
+    } catch (...) {
+      dfree(g); dfree(e); dfree(d); dfree(bases);
+      throw;
+    }
+    dfree(g); dfree(e); dfree(d); dfree(bases);
+  }
+
+  void debug_field(int op, const uint32_t* a, const uint32_t* b, size_t n, uint32_t* out) override {
+    uint32_t *da, *db, *dout;
+    const size_t w = n * C::L32;
+    dalloc(&da, w); dalloc(&db, w); dalloc(&dout, w);
+    CK(cudaMemcpy(da, a, w * 4, cudaMemcpyHostToDevice));
+    CK(cudaMemcpy(db, b, w * 4, cudaMemcpyHostToDevice));
+    k_debug_field<C><<<(unsigned)cdiv(n, 128), 128>>>(op, da, db, n, dout);
+    CK(cudaGetLastError());
+    CK(cudaMemcpy(out, dout, w * 4, cudaMemcpyDeviceToHost));
+    dfree(da); dfree(db); dfree(dout);
+  }
+
+  void debug_ec(int op, const uint32_t* P, const uint32_t* Q, const uint32_t* z, size_t n, uint32_t* out) override {
+    uint32_t *dP, *dQ, *dz, *dout;
+    const size_t w = n * 2 * C::L32;
+    dalloc(&dP, w); dalloc(&dQ, w); dalloc(&dz, w); dalloc(&dout, w);
+    CK(cudaMemcpy(dP, P, w * 4, cudaMemcpyHostToDevice));
+    CK(cudaMemcpy(dQ, Q, w * 4, cudaMemcpyHostToDevice));
+    CK(cudaMemcpy(dz, z, w * 4, cudaMemcpyHostToDevice));
+    k_debug_ec<C><<<(unsigned)n, 1>>>(op, dP, dQ, dz, n, dout);  // one lane per warp: divergent EC paths
+    CK(cudaGetLastError());
+    CK(cudaMemcpy(out, dout, w * 4, cudaMemcpyDeviceToHost));
+    dfree(dP); dfree(dQ); dfree(dz); dfree(dout);
+  }
+
+  void debug_digits(int c, const uint32_t* scal, size_t n, int32_t* out) override {
+    const int nwin = num_windows(C::LAMBDA, c);
+    uint32_t* ds;
+    int32_t* dout;
+    dalloc(&ds, n * C::S);
+    dalloc(&dout, n * nwin);
+    CK(cudaMemcpy(ds, scal, n * C::S * 4, cudaMemcpyHostToDevice));
+    k_digits_debug<C><<<(unsigned)cdiv(n, 128), 128>>>(ds, n, c, nwin, dout);
+    CK(cudaGetLastError());
+    CK(cudaMemcpy(out, dout, n * nwin * 4, cudaMemcpyDeviceToHost));
+    dfree(ds); dfree(dout);
+  }
+
+  long count_nonempty(Shard& s) override {
+    unsigned long long* d;
+    dalloc(&d, 1);
+    CK(cudaMemsetAsync(d, 0, 8, s.stream));
+    k_count_nonempty<<<(unsigned)cdiv(s.F, 256), 256, 0, s.stream>>>(s.goff, s.F, d);
+    unsigned long long h = 0;
+    CK(cudaMemcpyAsync(&h, d, 8, cudaMemcpyDeviceToHost, s.stream));
+    CK(cudaStreamSynchronize(s.stream));
+    dfree(d);
+    return (long)h;
+  }
+
+  void to_affine(const uint32_t* in, size_t n, uint32_t* out, cudaStream_t st) override {
+    if (!n) return;
+    k_to_affine<C><<<(unsigned)cdiv(n, 64), 64, 0, st>>>(in, n, out);
+    CK(cudaGetLastError());
+  }
+};
+
+}  // namespace msmrt

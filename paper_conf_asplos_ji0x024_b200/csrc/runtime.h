@@ -1,0 +1,101 @@
+// Host runtime types shared by the C-ABI layer (engine.cu) and the per-curve kernel
+// translation units (curve_*.cu).  Host C++ only.
+#pragma once
+#include <cuda_runtime.h>
+
+#include <cstdint>
+#include <cstdio>
+#include <cstdlib>
+#include <vector>
+
+#include "../../include/msm.h"
+
+namespace msmrt {
+
+struct CudaError {
+  int code;
+};
+
+#define CK(call)                                                                         \
+  do {                                                                                   \
+    cudaError_t e_ = (call);                                                             \
+    if (e_ != cudaSuccess) {                                                             \
+      if (getenv("MSM_DEBUG")) fprintf(stderr, "msm: %s -> %s (%s:%d)\n", #call,        \
+                                       cudaGetErrorString(e_), __FILE__, __LINE__);      \
+      throw ::msmrt::CudaError{e_ == cudaErrorMemoryAllocation ? MSM_ERR_OOM : MSM_ERR_CUDA}; \
+    }                                                                                    \
+  } while (0)
+
+inline size_t cdiv(size_t a, size_t b) { return (a + b - 1) / b; }
+
+template <class T>
+void dalloc(T** p, size_t count) {
+  *p = nullptr;
+  if (count == 0) count = 1;
+  CK(cudaMalloc((void**)p, count * sizeof(T)));
+}
+template <class T>
+void dfree(T*& p) {
+  if (p) cudaFree(p);
+  p = nullptr;
+}
+
+enum { EV_START, EV_H2D, EV_SORT, EV_ACC, EV_FIX, EV_RED, EV_COMB, EV_END, EV_COUNT };
+
+// One device's share of a context: its points, scratch and stream.
+struct Shard {
+  int dev = 0;
+  size_t off = 0, n = 0;
+  cudaStream_t stream = nullptr;
+  cudaEvent_t ev[EV_COUNT] = {};
+  // configuration (depends on c)
+  int c = 0, nwin = 0;
+  uint32_t NB = 0;     // buckets per window incl. bucket 0 = 2^(c-1) + 1
+  size_t F = 0;        // flat buckets = nwin * NB
+  uint32_t acc_threads = 0, slice = 0;
+  uint32_t seg = 0, nseg = 0;
+  size_t ntiles = 0;
+  // device buffers
+  uint32_t *pts = nullptr, *scal = nullptr, *counts = nullptr, *goff = nullptr, *cursor = nullptr,
+           *sorted = nullptr, *buckets = nullptr, *carry_pts = nullptr, *segA = nullptr, *segB = nullptr,
+           *W = nullptr, *partial = nullptr, *partials = nullptr, *tiles = nullptr, *err = nullptr,
+           *result = nullptr;
+  int32_t* carry_f = nullptr;
+  uint32_t* host_err = nullptr;  // pinned
+};
+
+struct Options {
+  int c = 0, threads = 0, seg = 0;
+};
+
+// Per-curve kernels behind a virtual interface (one instance per curve, curve_*.cu).
+struct CurveOps {
+  virtual ~CurveOps() {}
+  virtual int L32() const = 0;
+  virtual int S() const = 0;
+  virtual int lambda() const = 0;
+  virtual int PW() const = 0;
+  virtual int XW() const = 0;
+  virtual void points_to_mont(Shard& s, const uint32_t* in_dev, size_t n) = 0;
+  virtual void configure(const Options& o, Shard& s, int c) = 0;
+  virtual void free_scratch(Shard& s) = 0;
+  // enqueue a2..a6 on s.stream for the shard's scalars; the partial ends in s.partial.
+  // Returns the number of kernels launched.
+  virtual int enqueue_pipeline(Shard& s, const uint32_t* scal_dev, bool timed) = 0;
+  virtual void enqueue_finalize(const uint32_t* partials_dev, int count, uint32_t* result_dev, cudaStream_t st) = 0;
+  virtual void gen_points(const uint32_t* e0, const uint32_t* delta, size_t n, uint32_t* out) = 0;
+  virtual void debug_field(int op, const uint32_t* a, const uint32_t* b, size_t n, uint32_t* out) = 0;
+  virtual void debug_ec(int op, const uint32_t* P, const uint32_t* Q, const uint32_t* z, size_t n, uint32_t* out) = 0;
+  virtual void debug_digits(int c, const uint32_t* scal, size_t n, int32_t* out) = 0;
+  virtual void to_affine(const uint32_t* in_dev, size_t n, uint32_t* out_dev, cudaStream_t st) = 0;
+  virtual long count_nonempty(Shard& s) = 0;
+};
+
+inline int num_windows(int lambda, int c) { return lambda / c + 1; }
+
+CurveOps* make_ops_bn254();
+CurveOps* make_ops_bls12_377();
+CurveOps* make_ops_bls12_381();
+CurveOps* make_ops_mnt4_753();
+
+}  // namespace msmrt

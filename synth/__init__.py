@@ -114,3 +114,42 @@ def pattern_scalars(r: int, n: int, seed: int, kind: str) -> np.ndarray:
     else:
         raise ValueError(kind)
     return ints_to_words(vals, S)
+
+
+SCALAR_CHUNK = 1 << 20
+
+
+def scalars_range(r: int, start: int, count: int, seed: int) -> np.ndarray:
+    """Rows [start, start+count) of an arbitrarily long uniform scalar vector: chunk t of
+    SCALAR_CHUNK rows is drawn from seed (seed, t), so any slice (a rank's shard) is
+    generated independently and identically for every world size."""
+    lam = r.bit_length()
+    S = (lam + 31) // 32
+    out = np.empty((count, S), dtype=np.uint32)
+    t0 = start // SCALAR_CHUNK
+    t1 = (start + count + SCALAR_CHUNK - 1) // SCALAR_CHUNK
+    for t in range(t0, t1):
+        lo = max(start, t * SCALAR_CHUNK)
+        hi = min(start + count, (t + 1) * SCALAR_CHUNK)
+        if hi <= lo:
+            continue
+        chunk = scalars(r, SCALAR_CHUNK, (seed * 1000003 + t) & 0x7FFFFFFFFFFFFFFF)
+        out[lo - start:hi - start] = chunk[lo - t * SCALAR_CHUNK:hi - t * SCALAR_CHUNK]
+    return out
+
+
+def progression_offset(r: int, e0: int, delta: int, off: int) -> int:
+    """e_off = e0 + off*delta mod r: the first point scalar of a shard starting at `off`
+    (input bookkeeping for the generator, not curve arithmetic)."""
+    return (e0 + off * delta) % r
+
+
+# Scalar-field orders r (bit length = λ, PAPER.md Table 1): the range of the uniform scalar
+# draw.  Constants of the input recipe, not arithmetic; the oracle keeps its own copy in
+# oracle/curves.py and the library its own in csrc/params.h.
+CURVE_ORDERS = {
+    "bn254": 0x30644e72e131a029b85045b68181585d2833e84879b9709143e1f593f0000001,
+    "bls12_377": 0x12ab655e9a2ca55660b44d1e5c37b00159aa76fed00000010a11800000000001,
+    "bls12_381": 0x73eda753299d7d483339d80809a1d80553bda402fffe5bfeffffffff00000001,
+    "mnt4_753": 0x01c4c62d92c41110229022eee2cdadb7f997505b8fafed5eb7e8f96c97d87307fdb925e8a0ed8d99d124d9a15af79db26c5c28c859a99b3eebca9429212636b9dff97634993aa4d6c381bc3f0057974ea099170fa13a4fd90776e240000001,
+}
