@@ -21,6 +21,10 @@ typedef unsigned long long u64;
 
 #define DEVI __device__ __forceinline__
 
+#ifndef MSM_FMUL_CARRY_LATE
+#define MSM_FMUL_CARRY_LATE 0
+#endif
+
 // One IMAD.WIDE.U32 (a*b + c, 64-bit addend).  The product is an explicit PTX
 // mul.wide.u32 and the add is C++: ptxas then emits a clean IMAD.WIDE.U32 chain.
 // (An inline-asm mad.wide.u32 chain gets re-associated into IMAD.WIDE + IADD3 trees,
@@ -51,9 +55,18 @@ DEVI void fmul(uint32_t* r, const uint32_t* a, const uint32_t* b) {
       const int lo = k - L + 1 > 0 ? k - L + 1 : 0;
       const int hiA = k < L - 1 ? k : L - 1;
       const int hiM = (k - 1) < (L - 1) ? k - 1 : L - 1;
+#if MSM_FMUL_CARRY_LATE
+      // a*b column chain starts from 0 (independent of earlier columns: ILP across
+      // columns); the carry is added after the chain (one 64-bit add)
+      u64 accA = 0, accM = cM;
+#pragma unroll
+      for (int i = lo; i <= hiA; i++) accA = mad_wide(a[i], b[k - i], accA);
+      accA += cA;
+#else
       u64 accA = cA, accM = cM;
 #pragma unroll
       for (int i = lo; i <= hiA; i++) accA = mad_wide(a[i], b[k - i], accA);
+#endif
 #pragma unroll
       for (int i = lo; i <= hiM; i++) accM = mad_wide(m[i], C::P(k - i), accM);
       if (k < L) {

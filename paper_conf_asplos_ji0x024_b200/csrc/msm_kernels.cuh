@@ -16,6 +16,13 @@ namespace msmk {
 
 constexpr uint32_t SIGN_BIT = 0x80000000u;
 
+#ifndef MSM_ACC_MINB
+#define MSM_ACC_MINB 1  // min resident 128-thread blocks per SM for k_accumulate (register cap)
+#endif
+#ifndef MSM_SEG_MINB
+#define MSM_SEG_MINB 1
+#endif
+
 template <class C>
 struct Layout {
   static constexpr int PW = ((2 * C::L + 3) / 4) * 4;  // words per stored affine point
@@ -344,7 +351,7 @@ DEVI uint32_t find_bucket(const uint32_t* __restrict__ goff, uint32_t F, uint32_
 }
 
 template <class C>
-__global__ void __launch_bounds__(128) k_accumulate(const uint32_t* __restrict__ pts, const uint32_t* __restrict__ sorted,
+__global__ void __launch_bounds__(128, MSM_ACC_MINB) k_accumulate(const uint32_t* __restrict__ pts, const uint32_t* __restrict__ sorted,
                                                     const uint32_t* __restrict__ goff, uint32_t F, uint32_t slice,
                                                     uint32_t* __restrict__ buckets, uint32_t* __restrict__ carry_pts,
                                                     int32_t* __restrict__ carry_f, uint32_t nthreads) {
@@ -439,7 +446,7 @@ DEVI void xyzz_mul_small(Xyzz<C>& R, const Xyzz<C>& A, uint32_t k, int bits) {
 }
 
 template <class C>
-__global__ void __launch_bounds__(128) k_bucket_segments(const uint32_t* __restrict__ buckets, const uint32_t* __restrict__ goff,
+__global__ void __launch_bounds__(128, MSM_SEG_MINB) k_bucket_segments(const uint32_t* __restrict__ buckets, const uint32_t* __restrict__ goff,
                                                          int nwin, uint32_t NB, uint32_t seg, uint32_t nseg,
                                                          uint32_t* __restrict__ out) {
   constexpr int XW = Layout<C>::XW;

@@ -16,7 +16,7 @@ import numpy as np
 
 _LIB = None
 _HERE = os.path.dirname(os.path.abspath(__file__))
-LIB_PATH = os.path.join(_HERE, "libmsm.so")
+LIB_PATH = os.environ.get("MSM_LIB") or os.path.join(_HERE, "libmsm.so")  # MSM_LIB: A/B variant builds
 
 CURVE_IDS = {"bn254": 0, "bls12_377": 1, "bls12_381": 2, "mnt4_753": 3}
 

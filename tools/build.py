@@ -28,12 +28,12 @@ def newest_header():
     return max(os.path.getmtime(h) for h in hs)
 
 
-def compile_one(src, force):
-    obj = os.path.join(BUILD, os.path.basename(src).replace(".cu", ".o"))
+def compile_one(src, force, build_dir=BUILD, defines=()):
+    obj = os.path.join(build_dir, os.path.basename(src).replace(".cu", ".o"))
     log = obj + ".log"
     if not force and os.path.exists(obj) and os.path.getmtime(obj) >= max(os.path.getmtime(src), newest_header()):
         return obj, "cached"
-    cmd = [NVCC] + FLAGS + ["-c", src, "-o", obj]
+    cmd = [NVCC] + FLAGS + [f"-D{d}" for d in defines] + ["-c", src, "-o", obj]
     r = subprocess.run(cmd, capture_output=True, text=True)
     with open(log, "w") as f:
         f.write(" ".join(cmd) + "\n" + r.stdout + r.stderr)
@@ -42,34 +42,50 @@ def compile_one(src, force):
     return obj, "built"
 
 
-def build(jobs=8, force=False, verbose=True):
-    os.makedirs(BUILD, exist_ok=True)
+def build(jobs=8, force=False, verbose=True, only=None, defines=(), out=OUT, build_dir=BUILD):
+    """only: curve TU names to (re)compile (others reuse build_dir objects: dev/variants);
+    defines: extra -D macros (kernel variants for A/B runs)."""
+    os.makedirs(build_dir, exist_ok=True)
     srcs = sorted(glob.glob(os.path.join(CSRC, "*.cu")))
+    if only:
+        keep = [s for s in srcs if "curve_" not in s or any(o in s for o in only)]
+        stale = [s for s in srcs if s not in keep]
+        srcs = keep
+        for s_ in stale:  # reuse objects from the main build dir
+            o = os.path.join(build_dir, os.path.basename(s_).replace(".cu", ".o"))
+            src_o = os.path.join(BUILD, os.path.basename(s_).replace(".cu", ".o"))
+            if build_dir != BUILD and not os.path.exists(o):
+                import shutil
+                shutil.copy(src_o, o)
     # MNT4-753 is the slowest TU: start it first
     srcs.sort(key=lambda s: 0 if "mnt4" in s else 1)
     with cf.ThreadPoolExecutor(max_workers=jobs) as ex:
-        res = list(ex.map(lambda s: compile_one(s, force), srcs))
-    objs = [o for o, _ in res]
+        res = list(ex.map(lambda s: compile_one(s, force, build_dir, defines), srcs))
+    objs = sorted(glob.glob(os.path.join(build_dir, "*.o")))
     if verbose:
         for o, st in res:
             print(f"  {os.path.basename(o)}: {st}")
-    if force or not os.path.exists(OUT) or any(os.path.getmtime(o) > os.path.getmtime(OUT) for o in objs):
-        cmd = [NVCC, "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-o", OUT] + objs
+    if force or not os.path.exists(out) or any(os.path.getmtime(o) > os.path.getmtime(out) for o in objs):
+        cmd = [NVCC, "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-o", out] + objs
         r = subprocess.run(cmd, capture_output=True, text=True)
         if r.returncode != 0:
             raise RuntimeError("link failed:\n" + r.stderr[-4000:])
     if verbose:
-        print("built", OUT)
-    return OUT
+        print("built", out)
+    return out
 
 
 if __name__ == "__main__":
     ap = argparse.ArgumentParser()
     ap.add_argument("-j", type=int, default=8)
     ap.add_argument("--force", action="store_true")
+    ap.add_argument("--only", default="", help="comma-separated curve TUs to compile (dev)")
+    ap.add_argument("-D", action="append", default=[], help="extra macro for a variant build")
+    ap.add_argument("--out", default=OUT)
+    ap.add_argument("--build-dir", default=BUILD)
     a = ap.parse_args()
     try:
-        build(a.j, a.force)
+        build(a.j, a.force, only=[o for o in a.only.split(",") if o], defines=a.D, out=a.out, build_dir=a.build_dir)
     except RuntimeError as e:
         print(e, file=sys.stderr)
         sys.exit(1)
