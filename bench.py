@@ -43,6 +43,16 @@ def imad_slots_per_mult(L):
     return 2 * L * L * 2 + L
 
 
+def imad_slots_per_sqr(L):
+    """Squaring: L(L+1)/2 a*a products + L^2 m*p products (2 slots each) + L m_k."""
+    return 2 * (L * (L + 1) // 2 + L * L) + L
+
+
+def imad_slots_per_pacc(L):
+    """PACC (Alg. 4) = 8 multiplications + 2 squarings (PP = P^2, V = R^2)."""
+    return 8 * imad_slots_per_mult(L) + 2 * imad_slots_per_sqr(L)
+
+
 def peaks():
     path = os.path.join(ROOT, "MEASURED_PEAKS.json")
     try:
@@ -186,6 +196,7 @@ def main():
 
     import synth
     from paper_conf_asplos_ji0x024_b200 import msm
+    from paper_conf_asplos_ji0x024_b200.dist import gather_and_finalize, shard_bounds
 
     ws, rank, local = dist_env()
     assert ws == args.gpus, f"--gpus {args.gpus} but WORLD_SIZE {ws}"
@@ -198,8 +209,7 @@ def main():
     L32, S, lam, L, W = CURVE_INFO[curve]
     r = synth.CURVE_ORDERS[curve]
     n = 1 << args.log2n
-    off = n * rank // ws
-    n_g = n * (rank + 1) // ws - off
+    off, n_g = shard_bounds(n, ws, rank)
     seed = 20240427 + 3
     e0, delta = synth.point_seeds(r, seed)
 
@@ -220,16 +230,12 @@ def main():
     stream = torch.cuda.ExternalStream(ctx.stream(0), device=dev)
     pw = msm.partial_words(curve)
     partial = torch.zeros(pw, dtype=torch.int32, device=dev)
-    gathered = torch.zeros((ws, pw), dtype=torch.int32, device=dev)
 
     def step(scalars):
         if ws == 1:
             return ctx.run_words(scalars)
-        ctx.run_partial(scalars, partial)
-        torch.distributed.all_gather_into_tensor(gathered, partial)
-        if rank == 0:
-            return msm.finalize(curve, gathered, ws)
-        return None
+        ctx.run_partial(scalars, partial)          # a2..a6 on this rank's shard
+        return gather_and_finalize(curve, partial)  # a7: NCCL all-gather + msm_finalize on rank 0
 
     def barrier():
         torch.cuda.synchronize()
@@ -298,7 +304,7 @@ def main():
     st = stage[-1]
     nonempty = ctx.get_option(msm.OPT_NONEMPTY)
     pacc = int(st["entries"]) - int(nonempty)
-    slots = pacc * 10 * imad_slots_per_mult(L)
+    slots = pacc * imad_slots_per_pacc(L)
     acc_avg_ms = sum(acc_ms) / len(acc_ms)
     pk = peaks()
     sm_max = pk.get("sm_max_mhz", 1965.0)
@@ -333,7 +339,7 @@ def main():
         "latency_ms": {"mean": ms, "min": min(times), "max": max(times)},
         "roofline": {"kernel": "k_accumulate", "bound": "alu", "achieved": achieved / 1e12, "peak": peak_slots / 1e12,
                      "unit": "T IMAD-pipe slots/s", "frac": achieved / peak_slots, "traffic": None,
-                     "work": f"{pacc} PACC x 10 field mults x {imad_slots_per_mult(L)} slots",
+                     "work": f"{pacc} PACC x (8 mul x {imad_slots_per_mult(L)} + 2 sqr x {imad_slots_per_sqr(L)}) IMAD slots",
                      "peak_basis": f"148 SM x 64 IMAD slots/clk x {sm_max} MHz (clocks.max.sm); IMAD.WIDE = 2 slots (measured)",
                      "field_mults_per_s": pacc * 10 / (acc_avg_ms / 1e3)},
         "clocks": clocks,

@@ -60,6 +60,7 @@ enum {
   MSM_OPT_WINDOW_BITS = 1,    /* c in [2, 24]; 0 = automatic (cost model). Reallocates scratch. */
   MSM_OPT_ACC_THREADS = 2,    /* accumulation threads per device; 0 = automatic            */
   MSM_OPT_SEG_LEN = 3,        /* buckets per bucket-reduce segment; 0 = automatic          */
+  MSM_OPT_SORT = 4,           /* a3 variant: 0 = two-level binned sort (default), 1 = direct global atomics */
   MSM_OPT_NWIN = 101,         /* (get only) number of windows floor(lambda/c) + 1           */
   MSM_OPT_NONEMPTY = 102      /* (get only) non-empty buckets of the last run on device 0   */
 };

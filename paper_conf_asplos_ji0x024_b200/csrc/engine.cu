@@ -422,6 +422,10 @@ int msm_set_option(msm_context* ctx, int key, long value) {
       if (value < 0 || value > (1 << 20)) return MSM_ERR_ARG;
       ctx->opt.seg = (int)value;
       break;
+    case MSM_OPT_SORT:
+      if (value < 0 || value > 1) return MSM_ERR_ARG;
+      ctx->opt.sort = (int)value;
+      break;
     default:
       return MSM_ERR_ARG;
   }
@@ -434,6 +438,7 @@ long msm_get_option(msm_context* ctx, int key) {
     case MSM_OPT_WINDOW_BITS: return ctx->shards[0].c;
     case MSM_OPT_ACC_THREADS: return ctx->shards[0].acc_threads;
     case MSM_OPT_SEG_LEN: return ctx->shards[0].seg;
+    case MSM_OPT_SORT: return ctx->shards[0].sort_mode;
     case MSM_OPT_NWIN: return ctx->shards[0].nwin;
     case MSM_OPT_NONEMPTY: {
       long v = MSM_ERR_CUDA;

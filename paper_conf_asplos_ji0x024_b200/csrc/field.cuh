@@ -21,8 +21,8 @@ typedef unsigned long long u64;
 
 #define DEVI __device__ __forceinline__
 
-#ifndef MSM_FMUL_CARRY_LATE
-#define MSM_FMUL_CARRY_LATE 0
+#ifndef MSM_FSQR_AS_MUL
+#define MSM_FSQR_AS_MUL 0
 #endif
 
 // One IMAD.WIDE.U32 (a*b + c, 64-bit addend).  The product is an explicit PTX
@@ -43,74 +43,98 @@ struct Fp {
 };
 
 // ---- r = a*b*R^-1 mod p (lazy: result < 2p for inputs < 10p) ----
-template <class C>
-DEVI void fmul(uint32_t* r, const uint32_t* a, const uint32_t* b) {
+// Column k of the product scan (FIPS) accumulates, as IMAD.WIDE.U32 chains,
+//   the a*b terms  a_i b_{k-i}   (SQR: a_i (2a_{k-i}) for i < k-i, plus a_{k/2}^2)
+//   the m*p terms  m_i p_{k-i}   (i < k), then m_k = t_k n'_0 mod 2^W and + m_k p_0 (k < L).
+// A 64-bit accumulator holds MAXT = floor(2^64 / 2^(2W)) - 1 products of W-bit limbs plus
+// the incoming carry; a column with more terms splits them over two accumulators (a*b
+// and m*p) whose carries travel separately.  Edge columns (few terms) use one chain and
+// a cheaper epilogue.
+// One column as a template instance: every index below is a compile-time constant, so
+// the whole product scan is straight-line code on registers (no reliance on the loop
+// unroller, which gives up on 25 large column bodies and then spills m[] to local memory).
+template <class C, bool SQR, int K, bool PREV_SPLIT>
+DEVI void fmul_col(uint32_t* r, const uint32_t* a, const uint32_t* b, const uint32_t* a2, uint32_t* m, u64 cA, u64 cM) {
   constexpr int L = C::L, W = C::W;
   constexpr uint32_t MASK = (1u << W) - 1;
-  uint32_t m[L];
-  if constexpr (C::NACC == 2) {
-    u64 cA = 0, cM = 0;
+  constexpr int MAXT = (W == 30) ? 15 : (W == 29 ? 63 : 255);
+  constexpr int lo = K - L + 1 > 0 ? K - L + 1 : 0;
+  constexpr int hiA = K < L - 1 ? K : L - 1;
+  constexpr int hiM = (K - 1) < (L - 1) ? K - 1 : L - 1;
+  constexpr int nA = hiA - lo + 1;
+  constexpr int nM = (hiM >= lo ? hiM - lo + 1 : 0) + (K < L ? 1 : 0);
+  constexpr bool single = (C::NACC == 1) || (nA + nM <= MAXT);
+  u64 accA = cA;
+  if constexpr (SQR) {
 #pragma unroll
-    for (int k = 0; k < 2 * L - 1; k++) {
-      const int lo = k - L + 1 > 0 ? k - L + 1 : 0;
-      const int hiA = k < L - 1 ? k : L - 1;
-      const int hiM = (k - 1) < (L - 1) ? k - 1 : L - 1;
-#if MSM_FMUL_CARRY_LATE
-      // a*b column chain starts from 0 (independent of earlier columns: ILP across
-      // columns); the carry is added after the chain (one 64-bit add)
-      u64 accA = 0, accM = cM;
-#pragma unroll
-      for (int i = lo; i <= hiA; i++) accA = mad_wide(a[i], b[k - i], accA);
-      accA += cA;
-#else
-      u64 accA = cA, accM = cM;
-#pragma unroll
-      for (int i = lo; i <= hiA; i++) accA = mad_wide(a[i], b[k - i], accA);
-#endif
-#pragma unroll
-      for (int i = lo; i <= hiM; i++) accM = mad_wide(m[i], C::P(k - i), accM);
-      if (k < L) {
-        uint32_t s = (uint32_t)accA + (uint32_t)accM;
-        m[k] = (s * C::N0) & MASK;
-        accM = mad_wide(m[k], C::P(0), accM);
-        uint32_t loA = (uint32_t)accA & MASK, loM = (uint32_t)accM & MASK;
-        cA = accA >> W;
-        cM = (accM >> W) + ((loA + loM) >> W);
-      } else {
-        uint32_t s = ((uint32_t)accA & MASK) + ((uint32_t)accM & MASK);
-        r[k - L] = s & MASK;
-        cA = accA >> W;
-        cM = (accM >> W) + (s >> W);
-      }
-    }
-    r[L - 1] = (uint32_t)(cA + cM);
+    for (int i = lo; i < K - i; i++) accA = mad_wide(a[i], a2[K - i], accA);
+    if constexpr ((K & 1) == 0) accA = mad_wide(a[K >> 1], a[K >> 1], accA);
   } else {
-    u64 c = 0;
 #pragma unroll
-    for (int k = 0; k < 2 * L - 1; k++) {
-      const int lo = k - L + 1 > 0 ? k - L + 1 : 0;
-      const int hiA = k < L - 1 ? k : L - 1;
-      const int hiM = (k - 1) < (L - 1) ? k - 1 : L - 1;
-      u64 acc = c;
+    for (int i = lo; i <= hiA; i++) accA = mad_wide(a[i], b[K - i], accA);
+  }
+  u64 nA_carry, nM_carry;
+  if constexpr (single) {
+    u64 acc = PREV_SPLIT ? accA + cM : accA;
 #pragma unroll
-      for (int i = lo; i <= hiA; i++) acc = mad_wide(a[i], b[k - i], acc);
-#pragma unroll
-      for (int i = lo; i <= hiM; i++) acc = mad_wide(m[i], C::P(k - i), acc);
-      if (k < L) {
-        m[k] = ((uint32_t)acc * C::N0) & MASK;
-        acc = mad_wide(m[k], C::P(0), acc);
-      } else {
-        r[k - L] = (uint32_t)acc & MASK;
-      }
-      c = acc >> W;
+    for (int i = lo; i <= hiM; i++) acc = mad_wide(m[i], C::P(K - i), acc);
+    if constexpr (K < L) {
+      m[K] = ((uint32_t)acc * C::N0) & MASK;
+      acc = mad_wide(m[K], C::P(0), acc);
+    } else {
+      r[K - L] = (uint32_t)acc & MASK;
     }
-    r[L - 1] = (uint32_t)c;
+    nA_carry = acc >> W;
+    nM_carry = 0;
+  } else {
+    u64 accM = PREV_SPLIT ? cM : 0;
+#pragma unroll
+    for (int i = lo; i <= hiM; i++) accM = mad_wide(m[i], C::P(K - i), accM);
+    if constexpr (K < L) {
+      uint32_t s = (uint32_t)accA + (uint32_t)accM;
+      m[K] = (s * C::N0) & MASK;
+      accM = mad_wide(m[K], C::P(0), accM);
+      uint32_t loA = (uint32_t)accA & MASK, loM = (uint32_t)accM & MASK;
+      nA_carry = accA >> W;
+      nM_carry = (accM >> W) + ((loA + loM) >> W);
+    } else {
+      uint32_t s = ((uint32_t)accA & MASK) + ((uint32_t)accM & MASK);
+      r[K - L] = s & MASK;
+      nA_carry = accA >> W;
+      nM_carry = (accM >> W) + (s >> W);
+    }
+  }
+  if constexpr (K + 1 < 2 * L - 1) {
+    fmul_col<C, SQR, K + 1, !single>(r, a, b, a2, m, nA_carry, nM_carry);
+  } else {
+    r[L - 1] = (uint32_t)(single ? nA_carry : nA_carry + nM_carry);
   }
 }
 
-// r = a^2 (same contract as fmul)
+template <class C, bool SQR>
+DEVI void fmul_impl(uint32_t* r, const uint32_t* a, const uint32_t* b) {
+  constexpr int L = C::L;
+  uint32_t m[L];
+  uint32_t a2[L];
+  if constexpr (SQR) {
+#pragma unroll
+    for (int i = 0; i < L; i++) a2[i] = a[i] << 1;
+  }
+  fmul_col<C, SQR, 0, false>(r, a, b, a2, m, 0ull, 0ull);
+}
+
 template <class C>
-DEVI void fsqr(uint32_t* r, const uint32_t* a) { fmul<C>(r, a, a); }
+DEVI void fmul(uint32_t* r, const uint32_t* a, const uint32_t* b) { fmul_impl<C, false>(r, a, b); }
+
+// r = a^2 (same contract as fmul): L(L+1)/2 products instead of L^2
+template <class C>
+DEVI void fsqr(uint32_t* r, const uint32_t* a) {
+#if MSM_FSQR_AS_MUL
+  fmul_impl<C, false>(r, a, a);
+#else
+  fmul_impl<C, true>(r, a, a);
+#endif
+}
 
 // r = a + b (no reduction; bound(r) = bound(a) + bound(b) <= KMAX)
 template <class C>
@@ -304,7 +328,7 @@ __device__ __noinline__ void fmul_ni(uint32_t* r, const uint32_t* a, const uint3
 template <class C>
 DEVI void fmul_e(uint32_t* r, const uint32_t* a, const uint32_t* b) { fmul<C>(r, a, b); }
 template <class C>
-DEVI void fsqr_e(uint32_t* r, const uint32_t* a) { fmul_e<C>(r, a, a); }
+DEVI void fsqr_e(uint32_t* r, const uint32_t* a) { fsqr<C>(r, a); }
 
 // r = a^(p-2) = a^-1 (Montgomery form in and out; a != 0 mod p), Fermat (PAPER.md silent;
 // used only for the final affine normalisation)

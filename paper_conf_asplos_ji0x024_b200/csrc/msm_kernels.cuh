@@ -261,6 +261,39 @@ __device__ __forceinline__ uint32_t block_exclusive_scan(uint32_t v, uint32_t* s
   return warp_prefix + x - v;
 }
 
+static __global__ void k_bin_sort_impl(const uint32_t* __restrict__ binOff, const uint32_t* __restrict__ binIdx,
+                                       const uint16_t* __restrict__ binFine, int shift, uint32_t nbin, uint32_t NB,
+                                       uint32_t* __restrict__ goff, uint32_t* __restrict__ sorted) {
+  extern __shared__ uint32_t cnt[];
+  __shared__ uint32_t warp_sums[32];
+  const uint32_t fb = blockIdx.x;
+  const uint32_t j = fb / nbin, bin = fb % nbin;
+  const uint32_t e0 = binOff[fb], e1 = binOff[fb + 1];
+  const uint32_t nfine = 1u << shift;
+  for (uint32_t i = threadIdx.x; i < nfine; i += blockDim.x) cnt[i] = 0;
+  __syncthreads();
+  for (uint32_t e = e0 + threadIdx.x; e < e1; e += blockDim.x) atomicAdd(cnt + binFine[e], 1u);
+  __syncthreads();
+  // exclusive scan of cnt[0..nfine): each thread owns a contiguous chunk
+  const uint32_t per = (nfine + blockDim.x - 1) / blockDim.x;
+  const uint32_t c0 = threadIdx.x * per, c1 = min(c0 + per, nfine);
+  uint32_t sum = 0;
+  for (uint32_t i = c0; i < c1; i++) sum += cnt[i];
+  uint32_t run = block_exclusive_scan(sum, warp_sums, nullptr);
+  for (uint32_t i = c0; i < c1; i++) {
+    const uint32_t v = cnt[i];
+    cnt[i] = run;
+    const uint32_t b = (bin << shift) + i;
+    if (b < NB) goff[(size_t)j * NB + b] = e0 + run;
+    run += v;
+  }
+  __syncthreads();
+  for (uint32_t e = e0 + threadIdx.x; e < e1; e += blockDim.x) {
+    const uint32_t pos = atomicAdd(cnt + binFine[e], 1u);
+    sorted[e0 + pos] = binIdx[e];
+  }
+}
+
 static __global__ void k_scan_reduce(const uint32_t* __restrict__ counts, size_t F, uint32_t* __restrict__ tile_sums) {
   __shared__ uint32_t smem[32];
   size_t base = (size_t)blockIdx.x * SCAN_TILE + (size_t)threadIdx.x * SCAN_ITEMS;
@@ -310,6 +343,93 @@ static __global__ void k_scan_apply(const uint32_t* __restrict__ counts, size_t 
   }
 }
 
+// ---------------------------------------------------------------------------------------
+// a3, binned (default): two-level counting sort, the B200 form of the paper's hierarchical
+// bucket scatter (§3.2.1, Alg. 3).  With c up to 22 a window has 2^21 buckets,
+// far beyond shared memory (the paper's scheme stops at s = 14), so buckets are
+// grouped into coarse bins of 2^shift buckets (flat bin fb = j*nbin + (b >> shift),
+// nwin*nbin <= ~13K so a per-block bin histogram fits in shared memory):
+//   k_bin_count   per-block smem histogram over bins -> one global atomic per (block, bin)
+//   scan          bin offsets
+//   k_bin_scatter per-block smem ranks; one atomic per (block, bin) reserves a contiguous
+//                 run; entries (idx|sign, fine = b mod 2^shift) land in short runs per bin
+//   k_bin_sort    one block per bin: smem counting sort on `fine` (2^shift counters),
+//                 writes goff for the bin's buckets and the final sorted indices, all inside
+//                 the bin's own contiguous output range.
+constexpr int BIN_THREADS = 512;
+constexpr int BIN_PTS = 8;                       // points per thread per tile
+constexpr int BIN_TILE = BIN_THREADS * BIN_PTS;  // 4096 points per block
+
+template <class C>
+__global__ void __launch_bounds__(BIN_THREADS) k_bin_count(const uint32_t* __restrict__ scal, size_t n, int c, int nwin,
+                                                           int shift, uint32_t nbin, uint32_t* __restrict__ binCount,
+                                                           uint32_t* err) {
+  extern __shared__ uint32_t hist[];
+  const uint32_t FB = (uint32_t)nwin * nbin;
+  for (uint32_t i = threadIdx.x; i < FB; i += blockDim.x) hist[i] = 0;
+  __syncthreads();
+  const size_t base = (size_t)blockIdx.x * BIN_TILE;
+  bool bad = false;
+  for (int q = 0; q < BIN_PTS; q++) {
+    const size_t i = base + (size_t)q * BIN_THREADS + threadIdx.x;
+    if (i >= n) break;
+    ScalarReg<C> k;
+    load_scalar<C>(k, scal, i);
+    if (!scalar_in_range<C>(k)) { bad = true; continue; }
+    for_each_digit<C>(k, c, nwin, [&](int j, uint32_t b, bool) { atomicAdd(hist + (uint32_t)j * nbin + (b >> shift), 1u); });
+  }
+  if (bad) atomicOr(err, 4u);
+  __syncthreads();
+  for (uint32_t i = threadIdx.x; i < FB; i += blockDim.x)
+    if (hist[i]) atomicAdd(binCount + i, hist[i]);
+}
+
+template <class C>
+__global__ void __launch_bounds__(BIN_THREADS) k_bin_scatter(const uint32_t* __restrict__ scal, size_t n, int c, int nwin,
+                                                             int shift, uint32_t nbin, uint32_t* __restrict__ binCursor,
+                                                             uint32_t* __restrict__ binIdx, uint16_t* __restrict__ binFine) {
+  extern __shared__ uint32_t sm[];
+  const uint32_t FB = (uint32_t)nwin * nbin;
+  uint32_t* hist = sm;
+  uint32_t* base = sm + FB;
+  for (uint32_t i = threadIdx.x; i < FB; i += blockDim.x) hist[i] = 0;
+  __syncthreads();
+  const size_t tile = (size_t)blockIdx.x * BIN_TILE;
+  for (int q = 0; q < BIN_PTS; q++) {
+    const size_t i = tile + (size_t)q * BIN_THREADS + threadIdx.x;
+    if (i >= n) break;
+    ScalarReg<C> k;
+    load_scalar<C>(k, scal, i);
+    if (!scalar_in_range<C>(k)) continue;
+    for_each_digit<C>(k, c, nwin, [&](int j, uint32_t b, bool) { atomicAdd(hist + (uint32_t)j * nbin + (b >> shift), 1u); });
+  }
+  __syncthreads();
+  for (uint32_t i = threadIdx.x; i < FB; i += blockDim.x) {
+    const uint32_t h = hist[i];
+    base[i] = h ? atomicAdd(binCursor + i, h) : 0u;
+    hist[i] = 0;
+  }
+  __syncthreads();
+  const uint32_t fmask = (1u << shift) - 1u;
+  for (int q = 0; q < BIN_PTS; q++) {
+    const size_t i = tile + (size_t)q * BIN_THREADS + threadIdx.x;
+    if (i >= n) break;
+    ScalarReg<C> k;
+    load_scalar<C>(k, scal, i);
+    if (!scalar_in_range<C>(k)) continue;
+    for_each_digit<C>(k, c, nwin, [&](int j, uint32_t b, bool neg) {
+      const uint32_t fb = (uint32_t)j * nbin + (b >> shift);
+      const uint32_t pos = base[fb] + atomicAdd(hist + fb, 1u);
+      binIdx[pos] = (uint32_t)i | (neg ? SIGN_BIT : 0u);
+      binFine[pos] = (uint16_t)(b & fmask);
+    });
+  }
+}
+
+// k_bin_sort_impl (one block per flat bin, nfine = 2^shift <= 8192) is defined with the
+// scan helpers above.
+
+// ---------------------------------------------------------------------------------------
 // number of non-empty flat buckets (statistics only)
 static __global__ void k_count_nonempty(const uint32_t* __restrict__ goff, size_t F, unsigned long long* out) {
   size_t f = (size_t)blockIdx.x * blockDim.x + threadIdx.x;

@@ -30,6 +30,7 @@ struct Ops final : CurveOps {
   void free_scratch(Shard& s) override {
     dfree(s.counts); dfree(s.goff); dfree(s.cursor); dfree(s.sorted); dfree(s.buckets);
     dfree(s.carry_pts); dfree(s.carry_f); dfree(s.segA); dfree(s.segB); dfree(s.W); dfree(s.tiles);
+    dfree(s.binCount); dfree(s.binOff); dfree(s.binCursor); dfree(s.binIdx); dfree(s.binFine);
   }
 
   void configure(const Options& o, Shard& s, int c) override {
@@ -40,6 +41,14 @@ struct Ops final : CurveOps {
     s.NB = (1u << (c - 1)) + 1;
     s.F = (size_t)s.nwin * s.NB;
     s.ntiles = cdiv(s.F, SCAN_TILE);
+    s.sort_mode = o.sort;
+    s.shift = 0;
+    while (s.shift < 13 && (size_t)s.nwin * ((((size_t)1 << (c - 1)) >> s.shift) + 1) > 13000) s.shift++;
+    s.nbin = (uint32_t)((((size_t)1 << (c - 1)) >> s.shift) + 1);
+    s.FB = (uint32_t)s.nwin * s.nbin;
+    s.ntiles_bin = cdiv(s.FB, SCAN_TILE);
+    CK(cudaFuncSetAttribute(k_bin_count<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(s.FB * 4)));
+    CK(cudaFuncSetAttribute(k_bin_scatter<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(2 * s.FB * 4)));
     cudaDeviceProp prop;
     CK(cudaGetDeviceProperties(&prop, s.dev));
     const int sms = prop.multiProcessorCount;
@@ -73,7 +82,14 @@ struct Ops final : CurveOps {
     dalloc(&s.segA, (size_t)s.nwin * s.nseg * XW_);
     dalloc(&s.segB, (size_t)s.nwin * cdiv(s.nseg, 32) * XW_);
     dalloc(&s.W, (size_t)s.nwin * XW_);
-    dalloc(&s.tiles, s.ntiles + 1);
+    dalloc(&s.tiles, std::max(s.ntiles, s.ntiles_bin) + 1);
+    if (s.sort_mode == 0) {
+      dalloc(&s.binCount, s.FB);
+      dalloc(&s.binOff, s.FB + 1);
+      dalloc(&s.binCursor, s.FB);
+      dalloc(&s.binIdx, Mmax);
+      dalloc(&s.binFine, Mmax);
+    }
   }
 
   int enqueue_pipeline(Shard& s, const uint32_t* scal, bool timed) override {
@@ -82,18 +98,42 @@ struct Ops final : CurveOps {
     const size_t n = s.n;
     if (timed) CK(cudaEventRecord(s.ev[EV_H2D], st));
     // a2 + a3: digits, histogram, scan, scatter
-    CK(cudaMemsetAsync(s.counts, 0, s.F * sizeof(uint32_t), st));
-    if (n) {
-      k_digit_counts<C><<<(unsigned)cdiv(n, 256), 256, 0, st>>>(scal, n, s.c, s.nwin, s.NB, s.counts, s.err);
+    if (s.sort_mode == 0) {
+      CK(cudaMemsetAsync(s.binCount, 0, s.FB * sizeof(uint32_t), st));
+      const unsigned tiles = (unsigned)cdiv(std::max<size_t>(n, 1), BIN_TILE);
+      if (n) {
+        k_bin_count<C><<<tiles, BIN_THREADS, s.FB * 4, st>>>(scal, n, s.c, s.nwin, s.shift, s.nbin, s.binCount, s.err);
+        launches++;
+      }
+      k_scan_reduce<<<(unsigned)s.ntiles_bin, SCAN_THREADS, 0, st>>>(s.binCount, s.FB, s.tiles);
+      k_scan_tiles<<<1, 1024, 0, st>>>(s.tiles, s.ntiles_bin, s.binOff + s.FB);
+      k_scan_apply<<<(unsigned)s.ntiles_bin, SCAN_THREADS, 0, st>>>(s.binCount, s.FB, s.tiles, s.binOff, s.binCursor);
+      launches += 3;
+      if (n) {
+        k_bin_scatter<C><<<tiles, BIN_THREADS, 2 * s.FB * 4, st>>>(scal, n, s.c, s.nwin, s.shift, s.nbin, s.binCursor,
+                                                                  s.binIdx, s.binFine);
+        launches++;
+      }
+      CK(cudaMemcpyAsync(s.goff + s.F, s.binOff + s.FB, 4, cudaMemcpyDeviceToDevice, st));
+      const uint32_t nfine = 1u << s.shift;
+      const unsigned sort_threads = nfine >= 1024 ? 1024 : 256;
+      k_bin_sort_impl<<<s.FB, sort_threads, nfine * 4, st>>>(s.binOff, s.binIdx, s.binFine, s.shift, s.nbin, s.NB,
+                                                              s.goff, s.sorted);
       launches++;
-    }
-    k_scan_reduce<<<(unsigned)s.ntiles, SCAN_THREADS, 0, st>>>(s.counts, s.F, s.tiles);
-    k_scan_tiles<<<1, 1024, 0, st>>>(s.tiles, s.ntiles, s.goff + s.F);
-    k_scan_apply<<<(unsigned)s.ntiles, SCAN_THREADS, 0, st>>>(s.counts, s.F, s.tiles, s.goff, s.cursor);
-    launches += 3;
-    if (n) {
-      k_digit_scatter<C><<<(unsigned)cdiv(n, 256), 256, 0, st>>>(scal, n, s.c, s.nwin, s.NB, s.cursor, s.sorted);
-      launches++;
+    } else {
+      CK(cudaMemsetAsync(s.counts, 0, s.F * sizeof(uint32_t), st));
+      if (n) {
+        k_digit_counts<C><<<(unsigned)cdiv(n, 256), 256, 0, st>>>(scal, n, s.c, s.nwin, s.NB, s.counts, s.err);
+        launches++;
+      }
+      k_scan_reduce<<<(unsigned)s.ntiles, SCAN_THREADS, 0, st>>>(s.counts, s.F, s.tiles);
+      k_scan_tiles<<<1, 1024, 0, st>>>(s.tiles, s.ntiles, s.goff + s.F);
+      k_scan_apply<<<(unsigned)s.ntiles, SCAN_THREADS, 0, st>>>(s.counts, s.F, s.tiles, s.goff, s.cursor);
+      launches += 3;
+      if (n) {
+        k_digit_scatter<C><<<(unsigned)cdiv(n, 256), 256, 0, st>>>(scal, n, s.c, s.nwin, s.NB, s.cursor, s.sorted);
+        launches++;
+      }
     }
     CK(cudaGetLastError());
     if (timed) CK(cudaEventRecord(s.ev[EV_SORT], st));

@@ -55,17 +55,24 @@ struct Shard {
   uint32_t acc_threads = 0, slice = 0;
   uint32_t seg = 0, nseg = 0;
   size_t ntiles = 0;
+  // binned sort geometry (a3): flat bins fb = j*nbin + (b >> shift), FB = nwin*nbin
+  int sort_mode = 0, shift = 0;
+  uint32_t nbin = 0, FB = 0;
+  size_t ntiles_bin = 0;
   // device buffers
   uint32_t *pts = nullptr, *scal = nullptr, *counts = nullptr, *goff = nullptr, *cursor = nullptr,
            *sorted = nullptr, *buckets = nullptr, *carry_pts = nullptr, *segA = nullptr, *segB = nullptr,
            *W = nullptr, *partial = nullptr, *partials = nullptr, *tiles = nullptr, *err = nullptr,
            *result = nullptr;
   int32_t* carry_f = nullptr;
+  uint32_t *binCount = nullptr, *binOff = nullptr, *binCursor = nullptr, *binIdx = nullptr;
+  uint16_t* binFine = nullptr;
   uint32_t* host_err = nullptr;  // pinned
 };
 
 struct Options {
   int c = 0, threads = 0, seg = 0;
+  int sort = 0;  // 0: binned two-level sort (default), 1: direct global atomics (ablation)
 };
 
 // Per-curve kernels behind a virtual interface (one instance per curve, curve_*.cu).

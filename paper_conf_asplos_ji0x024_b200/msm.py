@@ -23,6 +23,7 @@ CURVE_IDS = {"bn254": 0, "bls12_377": 1, "bls12_381": 2, "mnt4_753": 3}
 OPT_WINDOW_BITS = 1
 OPT_ACC_THREADS = 2
 OPT_SEG_LEN = 3
+OPT_SORT = 4
 OPT_NWIN = 101
 OPT_NONEMPTY = 102
 

@@ -28,7 +28,7 @@ def run(lib, name, Ps, ks, c=None, ngpus=1):
     ctx = lib.Context(name, points_to_words(Ps, name), ngpus=ngpus, n=len(Ps))
     try:
         if c:
-            ctx.set_option(lib.OPT_WINDOW_BITS if hasattr(lib, "OPT_WINDOW_BITS") else 1, c)
+            ctx.set_option(lib.OPT_WINDOW_BITS, c)
         return ctx.run(synth.ints_to_words(ks, S_W[name]) if ks else np.zeros((0, S_W[name]), np.uint32))
     finally:
         ctx.close()
@@ -166,4 +166,43 @@ def test_device_resident_inputs(lib):
     assert ctx.run(St) == closed(name, ks, es)
     st = ctx.stats()
     assert st["h2d_ms"] >= 0 and st["accumulate_ms"] > 0
+    ctx.close()
+
+
+@pytest.mark.parametrize("name", ["bn254", "bls12_381"])
+@pytest.mark.parametrize("sort", [0, 1])
+@pytest.mark.parametrize("cbits", [4, 9, 13, 16])
+def test_sort_variants(lib, name, sort, cbits):
+    """a3 two-level binned sort (default) and direct-atomic sort (ablation) both give the
+    oracle's result and the oracle's bucket sums, for bin shifts 0..> 0."""
+    c = CURVES[name]
+    n = 700
+    Ps, es, _, _ = progression(name, n, 28)
+    ks = synth.words_to_ints(synth.scalars(c.r, n, 40 + cbits))
+    ctx = lib.Context(name, points_to_words(list(Ps), name), n=n)
+    ctx.set_option(lib.OPT_SORT, sort)
+    ctx.set_option(lib.OPT_WINDOW_BITS, cbits)
+    assert ctx.get_option(lib.OPT_SORT) == sort
+    sw = synth.ints_to_words(ks, S_W[name])
+    assert ctx.run(sw) == closed(name, ks, es)
+    if cbits <= 9:
+        Ws, Bs = ctx.windows(sw, with_buckets=True)
+        Bo = stages.bucket_sums(ks, list(Ps), cbits, c)
+        for j in range(len(Bo)):
+            for b in range(1, len(Bo[j])):
+                assert Bs[j][b] == ec.to_output(Bo[j][b]), (j, b)
+    ctx.close()
+
+
+def test_large_c_binned_sort(lib):
+    """c = 20..22 (the bench's windows): shift > 0 bins, many empty buckets at small n."""
+    name = "bls12_381"
+    c = CURVES[name]
+    n = 3000
+    Ps, es, _, _ = progression(name, n, 29)
+    ks = synth.words_to_ints(synth.scalars(c.r, n, 41))
+    ctx = lib.Context(name, points_to_words(list(Ps), name), n=n)
+    for cbits in (20, 22):
+        ctx.set_option(lib.OPT_WINDOW_BITS, cbits)
+        assert ctx.run(synth.ints_to_words(ks, 8)) == closed(name, ks, es), cbits
     ctx.close()
