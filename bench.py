@@ -200,11 +200,18 @@ def main():
 
     ws, rank, local = dist_env()
     assert ws == args.gpus, f"--gpus {args.gpus} but WORLD_SIZE {ws}"
-    torch.cuda.set_device(local)
-    dev = torch.device("cuda", local)
+    # MSM_BENCH_SHARE_DEVICE=1 (test only): every rank on cuda:0 and the gather over gloo
+    # with host partials, so the N > 1 path can be exercised on a one-GPU box.
+    share = os.environ.get("MSM_BENCH_SHARE_DEVICE") == "1"
+    torch.cuda.set_device(0 if share else local)
+    dev = torch.device("cuda", 0 if share else local)
+    coll_dev = torch.device("cpu") if share else dev
     if ws > 1:
         import torch.distributed as dist
-        dist.init_process_group("nccl", device_id=dev)
+        if share:
+            dist.init_process_group("gloo")
+        else:
+            dist.init_process_group("nccl", device_id=dev)
     curve = args.curve
     L32, S, lam, L, W = CURVE_INFO[curve]
     r = synth.CURVE_ORDERS[curve]
@@ -229,7 +236,7 @@ def main():
     setup_s = time.time() - t0
     stream = torch.cuda.ExternalStream(ctx.stream(0), device=dev)
     pw = msm.partial_words(curve)
-    partial = torch.zeros(pw, dtype=torch.int32, device=dev)
+    partial = torch.zeros(pw, dtype=torch.int32, device=coll_dev)
 
     def step(scalars):
         if ws == 1:
@@ -262,7 +269,7 @@ def main():
         barrier()
     times = [a.elapsed_time(b) for a, b in ev]
     my_ms = sum(times) / len(times)
-    t_all = torch.tensor([my_ms], dtype=torch.float64, device=dev)
+    t_all = torch.tensor([my_ms], dtype=torch.float64, device=coll_dev)
     if ws > 1:
         torch.distributed.all_reduce(t_all, op=torch.distributed.ReduceOp.MAX)
     ms = float(t_all.item())
@@ -281,7 +288,7 @@ def main():
             if ws > 1:
                 barrier()
             e_ms.append((time.perf_counter() - s0) * 1e3)
-        e_t = torch.tensor([sum(e_ms) / len(e_ms)], dtype=torch.float64, device=dev)
+        e_t = torch.tensor([sum(e_ms) / len(e_ms)], dtype=torch.float64, device=coll_dev)
         if ws > 1:
             torch.distributed.all_reduce(e_t, op=torch.distributed.ReduceOp.MAX)
         e2e_ms = float(e_t.item())

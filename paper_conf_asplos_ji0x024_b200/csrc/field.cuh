@@ -53,7 +53,11 @@ struct Fp {
 // One column as a template instance: every index below is a compile-time constant, so
 // the whole product scan is straight-line code on registers (no reliance on the loop
 // unroller, which gives up on 25 large column bodies and then spills m[] to local memory).
-template <class C, bool SQR, int K, bool PREV_SPLIT>
+// LAT (latency mode, for single-thread serial tails): the a*b products of a column form
+// two chains that start from 0 — independent of every earlier column — and the carry is
+// added afterwards, so a lone warp overlaps the columns instead of walking one long
+// dependency chain (2 extra ALU ops per column, irrelevant off the throughput path).
+template <class C, bool SQR, bool LAT, int K, bool PREV_SPLIT>
 DEVI void fmul_col(uint32_t* r, const uint32_t* a, const uint32_t* b, const uint32_t* a2, uint32_t* m, u64 cA, u64 cM) {
   constexpr int L = C::L, W = C::W;
   constexpr uint32_t MASK = (1u << W) - 1;
@@ -64,14 +68,34 @@ DEVI void fmul_col(uint32_t* r, const uint32_t* a, const uint32_t* b, const uint
   constexpr int nA = hiA - lo + 1;
   constexpr int nM = (hiM >= lo ? hiM - lo + 1 : 0) + (K < L ? 1 : 0);
   constexpr bool single = (C::NACC == 1) || (nA + nM <= MAXT);
-  u64 accA = cA;
-  if constexpr (SQR) {
+  u64 accA;
+  if constexpr (LAT) {
+    u64 e0 = 0, e1 = 0;
+    if constexpr (SQR) {
 #pragma unroll
-    for (int i = lo; i < K - i; i++) accA = mad_wide(a[i], a2[K - i], accA);
-    if constexpr ((K & 1) == 0) accA = mad_wide(a[K >> 1], a[K >> 1], accA);
+      for (int i = lo; i < K - i; i++) {
+        if ((i - lo) & 1) e1 = mad_wide(a[i], a2[K - i], e1);
+        else e0 = mad_wide(a[i], a2[K - i], e0);
+      }
+      if constexpr ((K & 1) == 0) e1 = mad_wide(a[K >> 1], a[K >> 1], e1);
+    } else {
+#pragma unroll
+      for (int i = lo; i <= hiA; i++) {
+        if ((i - lo) & 1) e1 = mad_wide(a[i], b[K - i], e1);
+        else e0 = mad_wide(a[i], b[K - i], e0);
+      }
+    }
+    accA = e0 + e1 + cA;
   } else {
+    accA = cA;
+    if constexpr (SQR) {
 #pragma unroll
-    for (int i = lo; i <= hiA; i++) accA = mad_wide(a[i], b[K - i], accA);
+      for (int i = lo; i < K - i; i++) accA = mad_wide(a[i], a2[K - i], accA);
+      if constexpr ((K & 1) == 0) accA = mad_wide(a[K >> 1], a[K >> 1], accA);
+    } else {
+#pragma unroll
+      for (int i = lo; i <= hiA; i++) accA = mad_wide(a[i], b[K - i], accA);
+    }
   }
   u64 nA_carry, nM_carry;
   if constexpr (single) {
@@ -105,13 +129,13 @@ DEVI void fmul_col(uint32_t* r, const uint32_t* a, const uint32_t* b, const uint
     }
   }
   if constexpr (K + 1 < 2 * L - 1) {
-    fmul_col<C, SQR, K + 1, !single>(r, a, b, a2, m, nA_carry, nM_carry);
+    fmul_col<C, SQR, LAT, K + 1, !single>(r, a, b, a2, m, nA_carry, nM_carry);
   } else {
     r[L - 1] = (uint32_t)(single ? nA_carry : nA_carry + nM_carry);
   }
 }
 
-template <class C, bool SQR>
+template <class C, bool SQR, bool LAT = false>
 DEVI void fmul_impl(uint32_t* r, const uint32_t* a, const uint32_t* b) {
   constexpr int L = C::L;
   uint32_t m[L];
@@ -120,11 +144,17 @@ DEVI void fmul_impl(uint32_t* r, const uint32_t* a, const uint32_t* b) {
 #pragma unroll
     for (int i = 0; i < L; i++) a2[i] = a[i] << 1;
   }
-  fmul_col<C, SQR, 0, false>(r, a, b, a2, m, 0ull, 0ull);
+  fmul_col<C, SQR, LAT, 0, false>(r, a, b, a2, m, 0ull, 0ull);
 }
 
 template <class C>
 DEVI void fmul(uint32_t* r, const uint32_t* a, const uint32_t* b) { fmul_impl<C, false>(r, a, b); }
+
+// latency-mode multiplication / squaring (serial tails: window combine, finalisation)
+template <class C>
+DEVI void fmul_lat(uint32_t* r, const uint32_t* a, const uint32_t* b) { fmul_impl<C, false, true>(r, a, b); }
+template <class C>
+DEVI void fsqr_lat(uint32_t* r, const uint32_t* a) { fmul_impl<C, true, true>(r, a, a); }
 
 // r = a^2 (same contract as fmul): L(L+1)/2 products instead of L^2
 template <class C>
@@ -325,10 +355,16 @@ __device__ __noinline__ void fmul_ni(uint32_t* r, const uint32_t* a, const uint3
 // a warp whose lanes diverge between a path with a call and one touching the stack
 // corrupts local memory — compute-sanitizer caught it.  Rule in this code base: calls to
 // __noinline__ functions only from warp-uniform control flow.)
-template <class C>
-DEVI void fmul_e(uint32_t* r, const uint32_t* a, const uint32_t* b) { fmul<C>(r, a, b); }
-template <class C>
-DEVI void fsqr_e(uint32_t* r, const uint32_t* a) { fsqr<C>(r, a); }
+template <class C, bool LAT = false>
+DEVI void fmul_e(uint32_t* r, const uint32_t* a, const uint32_t* b) {
+  if constexpr (LAT) fmul_lat<C>(r, a, b);
+  else fmul<C>(r, a, b);
+}
+template <class C, bool LAT = false>
+DEVI void fsqr_e(uint32_t* r, const uint32_t* a) {
+  if constexpr (LAT) fsqr_lat<C>(r, a);
+  else fsqr<C>(r, a);
+}
 
 // r = a^(p-2) = a^-1 (Montgomery form in and out; a != 0 mod p), Fermat (PAPER.md silent;
 // used only for the final affine normalisation)
@@ -339,8 +375,8 @@ __device__ __noinline__ void finv(uint32_t* r, const uint32_t* a) {
   for (int wi = C::L32 - 1; wi >= 0; wi--) {
     const uint32_t e = C::PM2c()[wi];
     for (int b = 31; b >= 0; b--) {
-      fmul_ni<C>(acc, acc, acc);
-      if ((e >> b) & 1u) fmul_ni<C>(acc, acc, a);
+      fsqr_lat<C>(acc, acc);
+      if ((e >> b) & 1u) fmul_lat<C>(acc, acc, a);
     }
   }
   fcopy<C>(r, acc);

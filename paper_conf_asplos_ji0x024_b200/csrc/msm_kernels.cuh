@@ -272,7 +272,19 @@ static __global__ void k_bin_sort_impl(const uint32_t* __restrict__ binOff, cons
   const uint32_t nfine = 1u << shift;
   for (uint32_t i = threadIdx.x; i < nfine; i += blockDim.x) cnt[i] = 0;
   __syncthreads();
-  for (uint32_t e = e0 + threadIdx.x; e < e1; e += blockDim.x) atomicAdd(cnt + binFine[e], 1u);
+  // loads batched U per thread (memory-level parallelism), then the smem atomics
+  constexpr int U = 8;
+  for (uint32_t e = e0 + threadIdx.x; e < e1; e += blockDim.x * U) {
+    uint32_t fv[U];
+#pragma unroll
+    for (int u = 0; u < U; u++) {
+      const uint32_t ee = e + u * blockDim.x;
+      fv[u] = ee < e1 ? (uint32_t)__ldg(binFine + ee) : 0xFFFFFFFFu;
+    }
+#pragma unroll
+    for (int u = 0; u < U; u++)
+      if (fv[u] != 0xFFFFFFFFu) atomicAdd(cnt + fv[u], 1u);
+  }
   __syncthreads();
   // exclusive scan of cnt[0..nfine): each thread owns a contiguous chunk
   const uint32_t per = (nfine + blockDim.x - 1) / blockDim.x;
@@ -288,9 +300,18 @@ static __global__ void k_bin_sort_impl(const uint32_t* __restrict__ binOff, cons
     run += v;
   }
   __syncthreads();
-  for (uint32_t e = e0 + threadIdx.x; e < e1; e += blockDim.x) {
-    const uint32_t pos = atomicAdd(cnt + binFine[e], 1u);
-    sorted[e0 + pos] = binIdx[e];
+  for (uint32_t e = e0 + threadIdx.x; e < e1; e += blockDim.x * U) {
+    uint32_t fv[U], iv[U];
+#pragma unroll
+    for (int u = 0; u < U; u++) {
+      const uint32_t ee = e + u * blockDim.x;
+      const bool ok = ee < e1;
+      fv[u] = ok ? (uint32_t)__ldg(binFine + ee) : 0xFFFFFFFFu;
+      iv[u] = ok ? __ldg(binIdx + ee) : 0u;
+    }
+#pragma unroll
+    for (int u = 0; u < U; u++)
+      if (fv[u] != 0xFFFFFFFFu) sorted[e0 + atomicAdd(cnt + fv[u], 1u)] = iv[u];
   }
 }
 
@@ -357,8 +378,8 @@ static __global__ void k_scan_apply(const uint32_t* __restrict__ counts, size_t 
 //                 writes goff for the bin's buckets and the final sorted indices, all inside
 //                 the bin's own contiguous output range.
 constexpr int BIN_THREADS = 512;
-constexpr int BIN_PTS = 8;                       // points per thread per tile
-constexpr int BIN_TILE = BIN_THREADS * BIN_PTS;  // 4096 points per block
+constexpr int BIN_PTS = 16;                      // points per thread per tile
+constexpr int BIN_TILE = BIN_THREADS * BIN_PTS;  // 8192 points per block: ~8 entries per bin per block
 
 template <class C>
 __global__ void __launch_bounds__(BIN_THREADS) k_bin_count(const uint32_t* __restrict__ scal, size_t n, int c, int nwin,
@@ -621,10 +642,14 @@ __global__ void k_window_combine(const uint32_t* __restrict__ W, int nwin, int c
   constexpr int XW = Layout<C>::XW;
   Xyzz<C> Q, B;
   load_xyzz<C>(Q, W + (size_t)(nwin - 1) * XW);
+  // single thread: inline latency-mode EC ops (no divergence, so no call hazard)
   for (int j = nwin - 2; j >= 0; j--) {
-    for (int s = 0; s < c; s++) xyzz_dbl_ni<C>(Q, Q);
+    for (int s = 0; s < c; s++) {
+      Xyzz<C> T = Q;
+      xyzz_dbl<C, true>(Q, T);
+    }
     load_xyzz<C>(B, W + (size_t)j * XW);
-    xyzz_add_ni<C>(Q, Q, B);
+    xyzz_add<C, true>(Q, Q, B);
   }
   store_xyzz<C>(partial, Q);
 }
@@ -638,7 +663,7 @@ __global__ void k_finalize(const uint32_t* __restrict__ partials, int count, uin
   xyzz_set_zero<C>(Q);
   for (int g = 0; g < count; g++) {
     load_xyzz<C>(B, partials + (size_t)g * XW);
-    xyzz_add_ni<C>(Q, Q, B);
+    xyzz_add<C, true>(Q, Q, B);
   }
   xyzz_to_affine_words<C>(result, result + C::L32, Q);
 }
