@@ -180,6 +180,8 @@ def main():
     ap.add_argument("--curve", default="bls12_381", choices=list(CURVE_INFO))
     ap.add_argument("--log2n", type=int, default=26)
     ap.add_argument("--window-bits", type=int, default=0)
+    ap.add_argument("--precompute", type=int, default=2, choices=[0, 1, 2],
+                    help="f3 window table (PAPER.md:147): 0 off, 1 on, 2 auto (library default)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--ref-sample", type=int, default=0)
     ap.add_argument("--no-e2e", action="store_true")
@@ -231,6 +233,8 @@ def main():
     ctx = msm.Context(curve, pts, ngpus=1, n=n_g)
     del pts
     torch.cuda.empty_cache()
+    if args.precompute != 2:
+        ctx.set_option(msm.OPT_PRECOMPUTE, args.precompute)
     if args.window_bits:
         ctx.set_option(msm.OPT_WINDOW_BITS, args.window_bits)
     setup_s = time.time() - t0
@@ -338,11 +342,13 @@ def main():
         "config": {"workload": f"{curve} G1 MSM n=2^{args.log2n} (BASELINE.json config C4)" if (curve, args.log2n) == ("bls12_381", 26)
                    else f"{curve} G1 MSM n=2^{args.log2n}",
                    "curve": curve, "n": n, "window_bits": st["window_bits"], "nwin": st["nwin"],
+                   "precompute": bool(st["precompute"]),
+                   "bucket_sets": 1 if st["precompute"] else st["nwin"],
                    "parallelism": f"point-sharded x{ws}" + (" + NCCL all-gather of partials" if ws > 1 else ""),
                    "scalars": "device-resident (HBM) for value; pinned host for e2e",
                    "l2": "inputs >> L2 (points %.1f GB + scalars %.1f GB per step); no flush needed" % (
                        n * (2 * L + 2) * 4 / 1e9, n * S * 4 / 1e9)},
-        "stages_ms": {k: round(v, 3) for k, v in st.items() if k.endswith("_ms")},
+        "stages_ms": {k: round(v, 3) for k, v in st.items() if k.endswith("_ms") and k != "table_ms"},
         "latency_ms": {"mean": ms, "min": min(times), "max": max(times)},
         "roofline": {"kernel": "k_accumulate", "bound": "alu", "achieved": achieved / 1e12, "peak": peak_slots / 1e12,
                      "unit": "T IMAD-pipe slots/s", "frac": achieved / peak_slots, "traffic": None,
@@ -352,6 +358,7 @@ def main():
         "clocks": clocks,
         "gpu_launches": int(st["acc_launches"]) * args.steps + (args.steps if ws > 1 else 0),
         "setup_s": round(setup_s, 2),
+        "table_build_s": round(st["table_ms"] / 1e3, 3) if st["precompute"] else 0.0,
     }
     if paper:
         line["paper_context"] = {"ms": paper, "hardware": f"{ws}x A100 80GB (DistMSM, PAPER.md Table 3)"}

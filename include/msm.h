@@ -61,7 +61,13 @@ enum {
   MSM_OPT_ACC_THREADS = 2,    /* accumulation threads per device; 0 = automatic            */
   MSM_OPT_SEG_LEN = 3,        /* buckets per bucket-reduce segment; 0 = automatic          */
   MSM_OPT_SORT = 4,           /* a3 variant: 0 = two-level binned sort (default), 1 = direct global atomics */
+  MSM_OPT_PRECOMPUTE = 5,     /* f3 window table 2^(jc) P_i: 0 off, 1 on,
+                                 2 auto (default: on when the table fits in device memory).
+                                 With it all windows share one bucket set; building the table
+                                 costs ~c*nwin doublings per point at create / option change;
+                                 get returns the mode in use (0/1).                          */
   MSM_OPT_NWIN = 101,         /* (get only) number of windows floor(lambda/c) + 1           */
+  MSM_OPT_NSETS = 103,        /* (get only) bucket sets: nwin, or 1 with the f3 table        */
   MSM_OPT_NONEMPTY = 102      /* (get only) non-empty buckets of the last run on device 0   */
 };
 
@@ -80,6 +86,8 @@ typedef struct {
   int acc_threads;      /* threads of k_accumulate                         */
   int acc_launches;     /* kernels launched by the last run (all devices)  */
   uint64_t entries;     /* sorted (bucket, point) entries = PACC + bucket starts, device 0 */
+  int precompute;       /* f3 table in use on device 0                     */
+  float table_ms;       /* time of the last f3 table build on device 0     */
 } msm_stats;
 
 typedef struct msm_context msm_context;
@@ -151,8 +159,10 @@ int msm_gen_points(int curve, const uint32_t* e0, const uint32_t* delta, size_t 
  *     per element (z1, z2 non-zero canonical); out: affine.
  *   msm_debug_digits: signed digits, out[i*nwin + j] (int32), nwin = floor(lambda/c)+1.
  *   msm_debug_windows: runs msm_run's pipeline on the context (ngpus == 1) and writes the
- *     window sums W_j (nwin affine points) to `windows`; if `buckets` is non-NULL also the
- *     bucket sums B_{j,b} for b = 0..2^(c-1) (nwin*(2^(c-1)+1) affine points, O where empty).
+ *     per-set sums W_s = sum_b b*B_{s,b} (nsets = msm_get_option(MSM_OPT_NSETS) affine
+ *     points: the window sums W_j without the f3 table, the whole MSM with it) to `windows`;
+ *     if `buckets` is non-NULL also the bucket sums B_{s,b} for b = 0..2^(c-1)
+ *     (nsets*(2^(c-1)+1) affine points, O where empty).
  */
 int msm_debug_field(int curve, int op, const uint32_t* a, const uint32_t* b, size_t n, uint32_t* out);
 int msm_debug_ec(int curve, int op, const uint32_t* P, const uint32_t* Q, const uint32_t* z, size_t n,

@@ -18,6 +18,14 @@ B_{j,b} = sum_{i : |d_ij| = b} sgn(d_ij) P_i                 (bucket-sum, PAPER.
 W_j     = sum_{b=1}^{2^(c-1)} b * B_{j,b}                     (bucket-reduce, PAPER.md:143, 161;
                                                              "2^i B_i" read as b*B_b, R12)
 Q       = sum_j 2^(j c) W_j  by Horner                        (window-reduce)
+
+With precomputation ("For a given point P_i, values such as 2^s P_i,
+2^{2s} P_i, and so on, are precomputed. As a result, in window j, the point P_i is
+replaced with 2^{js} P_i"; "bucket-reduce and window-reduce are commutative
+with precomputation") all windows share ONE bucket set:
+T_{j,i}  = 2^(j c) P_i                                        (table row j: c doublings of row j-1)
+B^pre_b  = sum_{(i,j) : |d_ij| = b} sgn(d_ij) T_{j,i}
+Q        = sum_{b=1}^{2^(c-1)} b * B^pre_b                    (one bucket-reduce, no window-reduce)
 """
 from . import ec
 
@@ -84,3 +92,36 @@ def window_combine(W, c, curve):
 
 def msm_staged(ks, Ps, c, curve):
     return window_combine(window_sums(bucket_sums(ks, Ps, c, curve), curve), c, curve)
+
+
+def precomputed_table(Ps, c, curve):
+    """T[j][i] = 2^(j c) P_i for j < nwin, each row c doublings of the previous one."""
+    nwin = num_windows(curve.lam, c)
+    T = [list(Ps)]
+    for _ in range(1, nwin):
+        row = []
+        for P in T[-1]:
+            for _ in range(c):
+                P = ec.double(P, curve)
+            row.append(P)
+        T.append(row)
+    return T
+
+
+def bucket_sums_precomputed(ks, Ps, c, curve):
+    """B^pre[b] (affine, None = O), b in 0..2^(c-1): one shared bucket set over all windows."""
+    T = precomputed_table(Ps, c, curve)
+    nb = (1 << (c - 1)) + 1
+    B = [None] * nb
+    for i, k in enumerate(ks):
+        for j, d in enumerate(signed_digits(k, curve.lam, c)):
+            if d == 0:
+                continue
+            Q = T[j][i] if d > 0 else ec.neg(T[j][i], curve)
+            B[abs(d)] = ec.add(B[abs(d)], Q, curve)
+    return B
+
+
+def msm_precomputed(ks, Ps, c, curve):
+    """Q = sum_b b * B^pre_b (a single bucket-reduce)."""
+    return window_sums([bucket_sums_precomputed(ks, Ps, c, curve)], curve)[0]

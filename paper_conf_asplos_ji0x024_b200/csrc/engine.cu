@@ -49,25 +49,67 @@ bool is_device_ptr(const void* p, int* dev) {
   return false;
 }
 
-// Pippenger cost model (field multiplications): per window n PACC (10 mults)
-// plus 2 PADD per bucket in the reduce (14 mults) over 2^(c-1) buckets.
-int choose_c(size_t n, int lambda) {
-  if (n == 0) return 8;
+// Pippenger cost model, in units of one PACC (10 field mults):
+//   per window n PACC ("ceil(lambda/s)(N + 2^{s+1})"), plus a sort cost per
+//   entry, plus the bucket reduce (2 PADD per bucket, measured ~4.4 PACC-equivalents per
+//   bucket on B200, r01 bench) over 2^(c-1) buckets per bucket set.  With the f3 table all
+//   windows share one bucket set, so larger c pays off.
+double plan_cost(size_t n, int lambda, int c, bool pre) {
+  const double nwin = num_windows(lambda, c);
+  const double sets = pre ? 1.0 : nwin;
+  return nwin * (double)n * 1.12 + sets * std::ldexp(1.0, c - 1) * 4.4;
+}
+
+// device bytes of the f3 table and of the per-run scratch for window size c
+size_t table_bytes(size_t n, int lambda, int c, int PW) { return (size_t)num_windows(lambda, c) * n * PW * 4; }
+size_t scratch_bytes(size_t n, int lambda, int c, int XW, bool pre) {
+  const size_t nwin = num_windows(lambda, c);
+  const size_t sets = pre ? 1 : nwin;
+  const size_t NB = ((size_t)1 << (c - 1)) + 1;
+  return n * nwin * 10 + sets * NB * ((size_t)XW * 4 + 12) + ((size_t)1 << 28);
+}
+
+// Chooses (c, pre) for one shard: opt.c / opt.pre when fixed; otherwise the cheapest
+// configuration whose device memory fits (the f3 table needs nwin*n < 2^31 entries too).
+void plan_shard(const Options& o, const Shard& s, int lambda, int PW, int XW, int* c_out, int* pre_out) {
+  size_t fr = 0, tot = 0;
+  CK(cudaSetDevice(s.dev));
+  CK(cudaMemGetInfo(&fr, &tot));
+  size_t held = 0;  // this shard's current table and scratch are freed before reallocation
+  if (s.table) held += table_bytes(s.n, lambda, s.table_c, PW);
+  if (s.sorted) held += scratch_bytes(s.n, lambda, s.c, XW, s.pre);
+  const double budget = 0.92 * (double)(fr + held) - (double)(2ull << 30);
+  auto fits = [&](int c, bool pre) {
+    double need = (double)scratch_bytes(s.n, lambda, c, XW, pre);
+    if (pre) need += (double)table_bytes(s.n, lambda, c, PW);
+    return need <= budget;
+  };
+  // sorted entries hold (table row j)*n + i in 31 bits
+  auto indexable = [&](int c) { return (double)num_windows(lambda, c) * (double)s.n < 2147483647.0; };
+  const int cmin = o.c > 0 ? o.c : 4, cmax = o.c > 0 ? o.c : 24;
   double best = 1e300;
-  int bc = 8;
-  for (int c = 4; c <= 22; c++) {
-    double cost = num_windows(lambda, c) * ((double)n * 10.0 + std::ldexp(1.0, c - 1) * 2 * 14.0);
-    if (cost < best) { best = cost; bc = c; }
+  int bc = o.c > 0 ? o.c : 8, bp = 0;
+  for (int pre = 0; pre <= 1; pre++) {
+    if ((o.pre == 0 && pre) || (o.pre == 1 && !pre)) continue;
+    for (int c = cmin; c <= cmax; c++) {
+      if (o.c <= 0 && c > 22 && !pre) continue;  // per-window bucket sets beyond 2^21
+      if (pre && !indexable(c)) continue;
+      if (o.pre == 2 && pre && !fits(c, true)) continue;
+      const double cost = s.n == 0 ? (double)c : plan_cost(s.n, lambda, c, pre);
+      if (cost < best) { best = cost; bc = c; bp = pre; }
+    }
   }
-  return bc;
+  if (best == 1e300) throw CudaError{MSM_ERR_ARG};  // forced table not indexable at this c
+  *c_out = bc;
+  *pre_out = bp;
 }
 
 CurveOps* ops_for(int curve) {
   switch (curve) {
-    case MSM_BN254: return make_ops_bn254();
-    case MSM_BLS12_377: return make_ops_bls12_377();
-    case MSM_BLS12_381: return make_ops_bls12_381();
-    case MSM_MNT4_753: return make_ops_mnt4_753();
+    case MSM_BN254: return make_ops_bn254 ? make_ops_bn254() : nullptr;
+    case MSM_BLS12_377: return make_ops_bls12_377 ? make_ops_bls12_377() : nullptr;
+    case MSM_BLS12_381: return make_ops_bls12_381 ? make_ops_bls12_381() : nullptr;
+    case MSM_MNT4_753: return make_ops_mnt4_753 ? make_ops_mnt4_753() : nullptr;
     default: return nullptr;
   }
 }
@@ -75,7 +117,10 @@ CurveOps* ops_for(int curve) {
 void destroy_shard(CurveOps* ops, Shard& s) {
   cudaSetDevice(s.dev);
   if (s.stream) cudaStreamSynchronize(s.stream);
-  if (ops) ops->free_scratch(s);
+  if (ops) {
+    ops->free_scratch(s);
+    ops->free_table(s);
+  }
   dfree(s.pts); dfree(s.scal); dfree(s.partial); dfree(s.partials); dfree(s.err); dfree(s.result);
   if (s.host_err) cudaFreeHost(s.host_err);
   s.host_err = nullptr;
@@ -87,8 +132,9 @@ void destroy_shard(CurveOps* ops, Shard& s) {
 
 int apply_window_bits(msm_context* ctx) {
   for (auto& s : ctx->shards) {
-    int c = ctx->opt.c > 0 ? ctx->opt.c : choose_c(s.n, ctx->ops->lambda());
-    ctx->ops->configure(ctx->opt, s, c);
+    int c = 0, pre = 0;
+    plan_shard(ctx->opt, s, ctx->ops->lambda(), ctx->ops->PW(), ctx->ops->XW(), &c, &pre);
+    ctx->ops->configure(ctx->opt, s, c, pre);
   }
   return MSM_OK;
 }
@@ -182,6 +228,8 @@ void collect_stats(msm_context* ctx) {
   uint32_t M = 0;
   cudaMemcpy(&M, s.goff + s.F, 4, cudaMemcpyDeviceToHost);
   st.entries = M;
+  st.precompute = s.pre;
+  st.table_ms = s.table_ms;
 }
 
 template <class F>
@@ -426,6 +474,10 @@ int msm_set_option(msm_context* ctx, int key, long value) {
       if (value < 0 || value > 1) return MSM_ERR_ARG;
       ctx->opt.sort = (int)value;
       break;
+    case MSM_OPT_PRECOMPUTE:
+      if (value < 0 || value > 2) return MSM_ERR_ARG;
+      ctx->opt.pre = (int)value;
+      break;
     default:
       return MSM_ERR_ARG;
   }
@@ -440,6 +492,8 @@ long msm_get_option(msm_context* ctx, int key) {
     case MSM_OPT_SEG_LEN: return ctx->shards[0].seg;
     case MSM_OPT_SORT: return ctx->shards[0].sort_mode;
     case MSM_OPT_NWIN: return ctx->shards[0].nwin;
+    case MSM_OPT_PRECOMPUTE: return ctx->shards[0].pre;
+    case MSM_OPT_NSETS: return ctx->shards[0].nset;
     case MSM_OPT_NONEMPTY: {
       long v = MSM_ERR_CUDA;
       guarded([&]() -> int { CK(cudaSetDevice(ctx->shards[0].dev)); v = ctx->ops->count_nonempty(ctx->shards[0]); return MSM_OK; });
@@ -512,9 +566,9 @@ int msm_debug_windows(msm_context* ctx, const uint32_t* scalars, uint32_t* windo
     if (e != MSM_OK) return e;
     const int L32 = ctx->ops->L32();
     uint32_t* dout;
-    dalloc(&dout, (size_t)s.nwin * 2 * L32);
-    ctx->ops->to_affine(s.W, s.nwin, dout, s.stream);
-    CK(cudaMemcpyAsync(windows, dout, (size_t)s.nwin * 2 * L32 * 4, cudaMemcpyDeviceToHost, s.stream));
+    dalloc(&dout, (size_t)s.nset * 2 * L32);
+    ctx->ops->to_affine(s.W, s.nset, dout, s.stream);
+    CK(cudaMemcpyAsync(windows, dout, (size_t)s.nset * 2 * L32 * 4, cudaMemcpyDeviceToHost, s.stream));
     CK(cudaStreamSynchronize(s.stream));
     dfree(dout);
     if (buckets) {

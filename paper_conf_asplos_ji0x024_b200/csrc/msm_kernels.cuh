@@ -124,6 +124,94 @@ __global__ void k_points_to_mont(uint32_t* __restrict__ pts, const uint32_t* __r
 }
 
 // ---------------------------------------------------------------------------------------
+// f3: precomputed window table ("in window j, the point P_i is replaced with
+// 2^{js} P_i"; :161 "bucket-reduce and window-reduce are commutative with precomputation").
+// Row j of the table is 2^c times row j-1, built at context creation in two passes per
+// chunk of points:
+//   k_pre_dbl   tmp[i] = 2^c * src[i]         (c XYZZ doublings, dbl-2008-s-1)
+//   k_pre_norm  dst[i] = affine(tmp[i])       (batch inversion: one Fermat inverse per
+//                                               PRE_K points, Montgomery's trick)
+// O (stored as x = y = 0) stays O.  Output values are < 2p (products), as PACC requires.
+constexpr int PRE_K = 32;
+
+template <class C>
+__global__ void __launch_bounds__(128) k_pre_dbl(const uint32_t* __restrict__ src, size_t cnt, int c,
+                                                 uint32_t* __restrict__ tmp) {
+  constexpr int XW = Layout<C>::XW;
+  const size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= cnt) return;
+  uint32_t x[C::L], y[C::L];
+  load_point<C>(x, y, src, (uint32_t)i);
+  Xyzz<C> A;
+  if (fis_zero<C, 2>(y)) xyzz_set_zero<C>(A);
+  else xyzz_from_affine<C>(A, x, y);
+  for (int s = 0; s < c; s++) {
+    Xyzz<C> T = A;
+    xyzz_dbl<C>(A, T);
+  }
+  store_xyzz<C>(tmp + i * XW, A);
+}
+
+// thread t normalises points [t*PRE_K, (t+1)*PRE_K) of tmp into dst; the prefix products
+// are parked in dst's records (PW >= L words) between the two sweeps.  Trip counts are
+// warp-uniform (tail lanes use d = 1) so the out-of-line finv is called convergently.
+template <class C>
+__global__ void __launch_bounds__(128) k_pre_norm(const uint32_t* __restrict__ tmp, size_t cnt,
+                                                  uint32_t* __restrict__ dst) {
+  constexpr int L = C::L, XW = Layout<C>::XW, PW = Layout<C>::PW;
+  const size_t t = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  const size_t i0 = t * PRE_K;
+  uint32_t acc[L], d[L], zz[L], zzz[L];
+  fset_one<C>(acc);
+  for (int k = 0; k < PRE_K; k++) {
+    const size_t i = i0 + k;
+    if (i < cnt) {
+      const uint32_t* q = tmp + i * XW;
+#pragma unroll
+      for (int w = 0; w < L; w++) { zz[w] = q[2 * L + w]; zzz[w] = q[3 * L + w]; }
+      fmul<C>(d, zz, zzz);
+      if (fis_zero<C, 2>(d)) fset_one<C>(d);
+      fmul<C>(acc, acc, d);
+#pragma unroll
+      for (int w = 0; w < L; w++) dst[i * PW + w] = acc[w];
+    }
+  }
+  uint32_t inv[L];
+  finv<C>(inv, acc);  // (prod d)^-1
+  for (int k = PRE_K - 1; k >= 0; k--) {
+    const size_t i = i0 + k;
+    if (i < cnt) {
+      const uint32_t* q = tmp + i * XW;
+      uint32_t X[L], Y[L], prev[L], ik[L], out[PW];
+#pragma unroll
+      for (int w = 0; w < L; w++) { X[w] = q[w]; Y[w] = q[L + w]; zz[w] = q[2 * L + w]; zzz[w] = q[3 * L + w]; }
+      if (k > 0) {
+#pragma unroll
+        for (int w = 0; w < L; w++) prev[w] = dst[(i - 1) * PW + w];
+      } else {
+        fset_one<C>(prev);
+      }
+      fmul<C>(ik, inv, prev);  // 1 / (ZZ * ZZZ)
+      fmul<C>(d, zz, zzz);
+      const bool inf = fis_zero<C, 2>(d);
+      if (!inf) fmul<C>(inv, inv, d);
+#pragma unroll
+      for (int w = 0; w < PW; w++) out[w] = 0;
+      if (!inf) {
+        uint32_t s[L];
+        fmul<C>(s, zzz, ik);     // 1/ZZ
+        fmul<C>(out, X, s);      // x = X / ZZ
+        fmul<C>(s, zz, ik);      // 1/ZZZ
+        fmul<C>(out + L, Y, s);  // y = Y / ZZZ
+      }
+      uint4* o4 = reinterpret_cast<uint4*>(dst + i * PW);
+#pragma unroll
+      for (int w = 0; w < PW / 4; w++) o4[w] = make_uint4(out[4 * w], out[4 * w + 1], out[4 * w + 2], out[4 * w + 3]);
+    }
+  }
+}
+
+// ---------------------------------------------------------------------------------------
 // a2: signed c-bit digits (R6):  nwin = floor(λ/c) + 1;  d_j = chunk_j + carry;
 //     for j < nwin-1: d_j > 2^(c-1) -> d_j -= 2^c, carry = 1.  Top digit never negated.
 template <class C>
@@ -191,30 +279,34 @@ DEVI void for_each_digit(const ScalarReg<C>& k, int c, int nwin, F&& f) {
   }
 }
 
-// histogram: counts[j*NB + b] += 1 for every non-zero digit.  err |= 4 for k >= r.
+// Flat bucket of digit (j, b): j*wstride + b, with wstride = NB (one bucket set per window)
+// or 0 (precomputed table, f3: all windows share one set).  The sorted entry of point i in
+// window j is (i + j*istride) | sign<<31 with istride = 0, or n (row j of the table).
+// histogram: counts[j*wstride + b] += 1 for every non-zero digit.  err |= 4 for k >= r.
 template <class C>
 __global__ void k_digit_counts(const uint32_t* __restrict__ scal, size_t n, int c, int nwin,
-                               uint32_t NB, uint32_t* __restrict__ counts, uint32_t* err) {
+                               uint32_t wstride, uint32_t* __restrict__ counts, uint32_t* err) {
   size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   ScalarReg<C> k;
   load_scalar<C>(k, scal, i);
   if (!scalar_in_range<C>(k)) { atomicOr(err, 4u); return; }
-  for_each_digit<C>(k, c, nwin, [&](int j, uint32_t b, bool) { atomicAdd(counts + (size_t)j * NB + b, 1u); });
+  for_each_digit<C>(k, c, nwin, [&](int j, uint32_t b, bool) { atomicAdd(counts + (size_t)j * wstride + b, 1u); });
 }
 
 // scatter: sorted[cursor[f]++] = i | sign << 31
 template <class C>
 __global__ void k_digit_scatter(const uint32_t* __restrict__ scal, size_t n, int c, int nwin,
-                                uint32_t NB, uint32_t* __restrict__ cursor, uint32_t* __restrict__ sorted) {
+                                uint32_t wstride, uint32_t istride, uint32_t* __restrict__ cursor,
+                                uint32_t* __restrict__ sorted) {
   size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
   if (i >= n) return;
   ScalarReg<C> k;
   load_scalar<C>(k, scal, i);
   if (!scalar_in_range<C>(k)) return;
   for_each_digit<C>(k, c, nwin, [&](int j, uint32_t b, bool neg) {
-    uint32_t pos = atomicAdd(cursor + (size_t)j * NB + b, 1u);
-    sorted[pos] = (uint32_t)i | (neg ? SIGN_BIT : 0u);
+    uint32_t pos = atomicAdd(cursor + (size_t)j * wstride + b, 1u);
+    sorted[pos] = ((uint32_t)i + (uint32_t)j * istride) | (neg ? SIGN_BIT : 0u);
   });
 }
 
@@ -383,10 +475,9 @@ constexpr int BIN_TILE = BIN_THREADS * BIN_PTS;  // 8192 points per block: ~8 en
 
 template <class C>
 __global__ void __launch_bounds__(BIN_THREADS) k_bin_count(const uint32_t* __restrict__ scal, size_t n, int c, int nwin,
-                                                           int shift, uint32_t nbin, uint32_t* __restrict__ binCount,
-                                                           uint32_t* err) {
+                                                           int shift, uint32_t FB, uint32_t wstride,
+                                                           uint32_t* __restrict__ binCount, uint32_t* err) {
   extern __shared__ uint32_t hist[];
-  const uint32_t FB = (uint32_t)nwin * nbin;
   for (uint32_t i = threadIdx.x; i < FB; i += blockDim.x) hist[i] = 0;
   __syncthreads();
   const size_t base = (size_t)blockIdx.x * BIN_TILE;
@@ -397,7 +488,7 @@ __global__ void __launch_bounds__(BIN_THREADS) k_bin_count(const uint32_t* __res
     ScalarReg<C> k;
     load_scalar<C>(k, scal, i);
     if (!scalar_in_range<C>(k)) { bad = true; continue; }
-    for_each_digit<C>(k, c, nwin, [&](int j, uint32_t b, bool) { atomicAdd(hist + (uint32_t)j * nbin + (b >> shift), 1u); });
+    for_each_digit<C>(k, c, nwin, [&](int j, uint32_t b, bool) { atomicAdd(hist + (uint32_t)j * wstride + (b >> shift), 1u); });
   }
   if (bad) atomicOr(err, 4u);
   __syncthreads();
@@ -407,10 +498,10 @@ __global__ void __launch_bounds__(BIN_THREADS) k_bin_count(const uint32_t* __res
 
 template <class C>
 __global__ void __launch_bounds__(BIN_THREADS) k_bin_scatter(const uint32_t* __restrict__ scal, size_t n, int c, int nwin,
-                                                             int shift, uint32_t nbin, uint32_t* __restrict__ binCursor,
+                                                             int shift, uint32_t FB, uint32_t wstride, uint32_t istride,
+                                                             uint32_t* __restrict__ binCursor,
                                                              uint32_t* __restrict__ binIdx, uint16_t* __restrict__ binFine) {
   extern __shared__ uint32_t sm[];
-  const uint32_t FB = (uint32_t)nwin * nbin;
   uint32_t* hist = sm;
   uint32_t* base = sm + FB;
   for (uint32_t i = threadIdx.x; i < FB; i += blockDim.x) hist[i] = 0;
@@ -422,7 +513,7 @@ __global__ void __launch_bounds__(BIN_THREADS) k_bin_scatter(const uint32_t* __r
     ScalarReg<C> k;
     load_scalar<C>(k, scal, i);
     if (!scalar_in_range<C>(k)) continue;
-    for_each_digit<C>(k, c, nwin, [&](int j, uint32_t b, bool) { atomicAdd(hist + (uint32_t)j * nbin + (b >> shift), 1u); });
+    for_each_digit<C>(k, c, nwin, [&](int j, uint32_t b, bool) { atomicAdd(hist + (uint32_t)j * wstride + (b >> shift), 1u); });
   }
   __syncthreads();
   for (uint32_t i = threadIdx.x; i < FB; i += blockDim.x) {
@@ -439,9 +530,9 @@ __global__ void __launch_bounds__(BIN_THREADS) k_bin_scatter(const uint32_t* __r
     load_scalar<C>(k, scal, i);
     if (!scalar_in_range<C>(k)) continue;
     for_each_digit<C>(k, c, nwin, [&](int j, uint32_t b, bool neg) {
-      const uint32_t fb = (uint32_t)j * nbin + (b >> shift);
+      const uint32_t fb = (uint32_t)j * wstride + (b >> shift);
       const uint32_t pos = base[fb] + atomicAdd(hist + fb, 1u);
-      binIdx[pos] = (uint32_t)i | (neg ? SIGN_BIT : 0u);
+      binIdx[pos] = ((uint32_t)i + (uint32_t)j * istride) | (neg ? SIGN_BIT : 0u);
       binFine[pos] = (uint16_t)(b & fmask);
     });
   }
@@ -493,13 +584,17 @@ DEVI uint32_t find_bucket(const uint32_t* __restrict__ goff, uint32_t F, uint32_
 
 template <class C>
 __global__ void __launch_bounds__(128, MSM_ACC_MINB) k_accumulate(const uint32_t* __restrict__ pts, const uint32_t* __restrict__ sorted,
-                                                    const uint32_t* __restrict__ goff, uint32_t F, uint32_t slice,
+                                                    const uint32_t* __restrict__ goff, uint32_t F,
                                                     uint32_t* __restrict__ buckets, uint32_t* __restrict__ carry_pts,
-                                                    int32_t* __restrict__ carry_f, uint32_t nthreads) {
+                                                    int32_t* __restrict__ carry_f, uint32_t nthreads,
+                                                    uint32_t* __restrict__ nlong) {
   constexpr int XW = Layout<C>::XW;
   const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+  if (t == 0) *nlong = 0;  // long-run list of k_fixup (same stream, later kernel)
   if (t >= nthreads) return;
+  // equal slices of the M entries actually present (M <= n*nwin: zero digits are skipped)
   const uint32_t M = __ldg(goff + F);
+  const uint32_t slice = M ? (M + nthreads - 1) / nthreads : 1u;
   const uint64_t e0l = (uint64_t)t * slice;
   if (e0l >= M) { carry_f[t] = -1; return; }
   const uint32_t e0 = (uint32_t)e0l;
@@ -539,14 +634,29 @@ DEVI void xyzz_select(Xyzz<C>& R, const Xyzz<C>& A, bool take) {
   else xyzz_set_zero<C>(R);
 }
 
-// run leaders sum the carries of their bucket and add them into buckets[f]
+// Carries of one bucket are consecutive (slices are in entry order).  Run leaders of short
+// runs (<= FIX_SHORT carries) add them serially into buckets[f]; longer runs (a bucket
+// spanning many slices: heavy buckets of skewed scalars, or a top window holding only the
+// carry digit) go to a list for k_fixup_long's block-wide tree.
+constexpr int FIX_SHORT = 8;
+constexpr int FIX_THREADS = 256;
+
 template <class C>
 __global__ void k_fixup(uint32_t* __restrict__ buckets, const uint32_t* __restrict__ carry_pts,
-                        const int32_t* __restrict__ carry_f, uint32_t nthreads) {
+                        const int32_t* __restrict__ carry_f, uint32_t nthreads,
+                        uint32_t* __restrict__ nlong, uint32_t* __restrict__ longs) {
   constexpr int XW = Layout<C>::XW;
   const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
   const int32_t f = t < nthreads ? carry_f[t] : -1;
-  const bool leader = f >= 0 && (t == 0 || carry_f[t - 1] != f);
+  bool leader = f >= 0 && (t == 0 || carry_f[t - 1] != f);
+  uint32_t R = 0;
+  if (leader) {
+    while (R <= FIX_SHORT && t + R < nthreads && carry_f[t + R] == f) R++;
+    if (R > FIX_SHORT) {
+      longs[atomicAdd(nlong, 1u)] = t;
+      leader = false;
+    }
+  }
   const unsigned mask = __ballot_sync(0xffffffffu, leader);
   if (!leader) return;
   Xyzz<C> s, b;
@@ -567,6 +677,62 @@ __global__ void k_fixup(uint32_t* __restrict__ buckets, const uint32_t* __restri
   __syncwarp(mask);
   xyzz_add_ni<C>(s, s, b);
   store_xyzz<C>(buckets + (size_t)f * XW, s);
+}
+
+// one block per long run (grid-stride over the list of run leaders): strided partial sums
+// while the run lasts (a bucket's carries are one contiguous run, so membership
+// carry_f[t] == f is exact for t >= t0), then a shared-memory tree; every lane calls the
+// adds (O operands where idle).
+template <class C>
+__global__ void __launch_bounds__(FIX_THREADS) k_fixup_long(uint32_t* __restrict__ buckets, const uint32_t* __restrict__ carry_pts,
+                                                            const int32_t* __restrict__ carry_f, uint32_t nthreads,
+                                                            const uint32_t* __restrict__ nlong, const uint32_t* __restrict__ longs) {
+  constexpr int XW = Layout<C>::XW;
+  extern __shared__ uint32_t red[];  // [FIX_THREADS][XW]
+  const uint32_t cnt = *nlong;
+  for (uint32_t q = blockIdx.x; q < cnt; q += gridDim.x) {
+    const uint32_t t0 = longs[q];
+    const int32_t f = carry_f[t0];
+    Xyzz<C> s, b;
+    xyzz_set_zero<C>(s);
+    for (uint32_t base = t0;; base += FIX_THREADS) {
+      const uint32_t u = base + threadIdx.x;
+      const bool in = u < nthreads && carry_f[u] == f;
+      if (!__syncthreads_or(in)) break;
+      if (in) load_xyzz<C>(b, carry_pts + (size_t)u * XW);
+      else xyzz_set_zero<C>(b);
+      xyzz_add_ni<C>(s, s, b);
+    }
+    store_xyzz<C>(red + threadIdx.x * XW, s);
+    __syncthreads();
+    for (int h = FIX_THREADS / 2; h >= 1; h >>= 1) {
+      if ((int)threadIdx.x < (h < 32 ? 32 : h)) {
+        if ((int)threadIdx.x < h) {
+          load_xyzz<C>(s, red + threadIdx.x * XW);
+          load_xyzz<C>(b, red + (threadIdx.x + h) * XW);
+        } else {
+          xyzz_set_zero<C>(s);
+          xyzz_set_zero<C>(b);
+        }
+        xyzz_add_ni<C>(s, s, b);
+      }
+      __syncthreads();
+      if ((int)threadIdx.x < h) store_xyzz<C>(red + threadIdx.x * XW, s);
+      __syncthreads();
+    }
+    if (threadIdx.x < 32) {
+      if (threadIdx.x == 0) {
+        load_xyzz<C>(s, red);
+        load_xyzz<C>(b, buckets + (size_t)f * XW);
+      } else {
+        xyzz_set_zero<C>(s);
+        xyzz_set_zero<C>(b);
+      }
+      xyzz_add_ni<C>(s, s, b);
+      if (threadIdx.x == 0) store_xyzz<C>(buckets + (size_t)f * XW, s);
+    }
+    __syncthreads();
+  }
 }
 
 // ---------------------------------------------------------------------------------------

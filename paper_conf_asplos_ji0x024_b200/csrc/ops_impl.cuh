@@ -31,27 +31,69 @@ struct Ops final : CurveOps {
     dfree(s.counts); dfree(s.goff); dfree(s.cursor); dfree(s.sorted); dfree(s.buckets);
     dfree(s.carry_pts); dfree(s.carry_f); dfree(s.segA); dfree(s.segB); dfree(s.W); dfree(s.tiles);
     dfree(s.binCount); dfree(s.binOff); dfree(s.binCursor); dfree(s.binIdx); dfree(s.binFine);
+    dfree(s.nlong); dfree(s.longs);
   }
 
-  void configure(const Options& o, Shard& s, int c) override {
+  void free_table(Shard& s) override {
+    dfree(s.table);
+    s.table_c = 0;
+  }
+
+  // f3: table[j][i] = 2^(j c) P_i for j < nwin (k_pre_dbl + k_pre_norm per chunk of points)
+  void build_table(Shard& s) {
+    const size_t n = s.n;
+    dalloc(&s.table, std::max<size_t>(1, (size_t)s.nwin * n) * PW_);
+    cudaEvent_t e0, e1;
+    CK(cudaEventCreate(&e0));
+    CK(cudaEventCreate(&e1));
+    CK(cudaEventRecord(e0, s.stream));
+    if (n) CK(cudaMemcpyAsync(s.table, s.pts, n * PW_ * 4, cudaMemcpyDeviceToDevice, s.stream));
+    const size_t chunk = std::min<size_t>(std::max<size_t>(n, 1), (size_t)1 << 22);
+    uint32_t* tmp = nullptr;
+    dalloc(&tmp, chunk * XW_);
+    for (int j = 1; j < s.nwin && n; j++) {
+      for (size_t off = 0; off < n; off += chunk) {
+        const size_t cnt = std::min(chunk, n - off);
+        const uint32_t* src = s.table + ((size_t)(j - 1) * n + off) * PW_;
+        uint32_t* dst = s.table + ((size_t)j * n + off) * PW_;
+        k_pre_dbl<C><<<(unsigned)cdiv(cnt, 128), 128, 0, s.stream>>>(src, cnt, s.c, tmp);
+        k_pre_norm<C><<<(unsigned)cdiv(cdiv(cnt, PRE_K), 128), 128, 0, s.stream>>>(tmp, cnt, dst);
+        CK(cudaGetLastError());
+      }
+    }
+    CK(cudaEventRecord(e1, s.stream));
+    CK(cudaStreamSynchronize(s.stream));
+    float ms = 0;
+    CK(cudaEventElapsedTime(&ms, e0, e1));
+    s.table_ms = ms;
+    cudaEventDestroy(e0);
+    cudaEventDestroy(e1);
+    dfree(tmp);
+    s.table_c = s.c;
+  }
+
+  void configure(const Options& o, Shard& s, int c, int pre) override {
     CK(cudaSetDevice(s.dev));
     free_scratch(s);
     s.c = c;
     s.nwin = num_windows(C::LAMBDA, c);
+    s.pre = pre;
+    s.nset = pre ? 1 : s.nwin;
     s.NB = (1u << (c - 1)) + 1;
-    s.F = (size_t)s.nwin * s.NB;
+    s.F = (size_t)s.nset * s.NB;
     s.ntiles = cdiv(s.F, SCAN_TILE);
     s.sort_mode = o.sort;
     s.shift = 0;
-    while (s.shift < 13 && (size_t)s.nwin * ((((size_t)1 << (c - 1)) >> s.shift) + 1) > 13000) s.shift++;
+    while (s.shift < 13 && (size_t)s.nset * ((((size_t)1 << (c - 1)) >> s.shift) + 1) > 13000) s.shift++;
     s.nbin = (uint32_t)((((size_t)1 << (c - 1)) >> s.shift) + 1);
-    s.FB = (uint32_t)s.nwin * s.nbin;
+    s.FB = (uint32_t)s.nset * s.nbin;
     s.ntiles_bin = cdiv(s.FB, SCAN_TILE);
     CK(cudaFuncSetAttribute(k_bin_count<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(s.FB * 4)));
     CK(cudaFuncSetAttribute(k_bin_scatter<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(2 * s.FB * 4)));
     cudaDeviceProp prop;
     CK(cudaGetDeviceProperties(&prop, s.dev));
     const int sms = prop.multiProcessorCount;
+    s.sms = sms;
     int bps = 0;
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_accumulate<C>, 128, 0));
     if (bps < 1) bps = 1;
@@ -67,11 +109,15 @@ struct Ops final : CurveOps {
     if (bps2 < 1) bps2 = 1;
     const size_t resident2 = (size_t)sms * bps2 * 128;
     const size_t nb = s.NB - 1;
-    uint32_t seg = o.seg > 0 ? (uint32_t)o.seg : 4;
-    if (o.seg <= 0)
-      while (seg < 4096 && (size_t)s.nwin * cdiv(nb, seg) > resident2) seg *= 2;
+    // one segment per resident thread (full occupancy, no tail wave); >= 4 buckets each
+    uint32_t seg = o.seg > 0 ? (uint32_t)o.seg : (uint32_t)std::max<size_t>(4, cdiv((size_t)s.nset * nb, resident2));
     s.seg = seg;
     s.nseg = (uint32_t)cdiv(nb, seg);
+    if (!pre) free_table(s);
+    else if (!s.table || s.table_c != c) {
+      free_table(s);
+      build_table(s);
+    }
     dalloc(&s.counts, s.F);
     dalloc(&s.goff, s.F + 1);
     dalloc(&s.cursor, s.F);
@@ -79,9 +125,12 @@ struct Ops final : CurveOps {
     dalloc(&s.buckets, s.F * XW_);
     dalloc(&s.carry_pts, (size_t)s.acc_threads * XW_);
     dalloc(&s.carry_f, s.acc_threads);
-    dalloc(&s.segA, (size_t)s.nwin * s.nseg * XW_);
-    dalloc(&s.segB, (size_t)s.nwin * cdiv(s.nseg, 32) * XW_);
-    dalloc(&s.W, (size_t)s.nwin * XW_);
+    dalloc(&s.nlong, 1);
+    dalloc(&s.longs, s.acc_threads);
+    CK(cudaFuncSetAttribute(k_fixup_long<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, FIX_THREADS * XW_ * 4));
+    dalloc(&s.segA, (size_t)s.nset * s.nseg * XW_);
+    dalloc(&s.segB, (size_t)s.nset * cdiv(s.nseg, 32) * XW_);
+    dalloc(&s.W, (size_t)s.nset * XW_);
     dalloc(&s.tiles, std::max(s.ntiles, s.ntiles_bin) + 1);
     if (s.sort_mode == 0) {
       dalloc(&s.binCount, s.FB);
@@ -96,13 +145,16 @@ struct Ops final : CurveOps {
     cudaStream_t st = s.stream;
     int launches = 0;
     const size_t n = s.n;
+    // flat-bucket / flat-bin stride per window and table-row stride (f3: one shared set)
+    const uint32_t ws = s.pre ? 0u : s.NB, wsb = s.pre ? 0u : s.nbin, istride = s.pre ? (uint32_t)n : 0u;
+    const uint32_t* pts = s.pre ? s.table : s.pts;
     if (timed) CK(cudaEventRecord(s.ev[EV_H2D], st));
     // a2 + a3: digits, histogram, scan, scatter
     if (s.sort_mode == 0) {
       CK(cudaMemsetAsync(s.binCount, 0, s.FB * sizeof(uint32_t), st));
       const unsigned tiles = (unsigned)cdiv(std::max<size_t>(n, 1), BIN_TILE);
       if (n) {
-        k_bin_count<C><<<tiles, BIN_THREADS, s.FB * 4, st>>>(scal, n, s.c, s.nwin, s.shift, s.nbin, s.binCount, s.err);
+        k_bin_count<C><<<tiles, BIN_THREADS, s.FB * 4, st>>>(scal, n, s.c, s.nwin, s.shift, s.FB, wsb, s.binCount, s.err);
         launches++;
       }
       k_scan_reduce<<<(unsigned)s.ntiles_bin, SCAN_THREADS, 0, st>>>(s.binCount, s.FB, s.tiles);
@@ -110,8 +162,8 @@ struct Ops final : CurveOps {
       k_scan_apply<<<(unsigned)s.ntiles_bin, SCAN_THREADS, 0, st>>>(s.binCount, s.FB, s.tiles, s.binOff, s.binCursor);
       launches += 3;
       if (n) {
-        k_bin_scatter<C><<<tiles, BIN_THREADS, 2 * s.FB * 4, st>>>(scal, n, s.c, s.nwin, s.shift, s.nbin, s.binCursor,
-                                                                  s.binIdx, s.binFine);
+        k_bin_scatter<C><<<tiles, BIN_THREADS, 2 * s.FB * 4, st>>>(scal, n, s.c, s.nwin, s.shift, s.FB, wsb, istride,
+                                                                  s.binCursor, s.binIdx, s.binFine);
         launches++;
       }
       CK(cudaMemcpyAsync(s.goff + s.F, s.binOff + s.FB, 4, cudaMemcpyDeviceToDevice, st));
@@ -123,7 +175,7 @@ struct Ops final : CurveOps {
     } else {
       CK(cudaMemsetAsync(s.counts, 0, s.F * sizeof(uint32_t), st));
       if (n) {
-        k_digit_counts<C><<<(unsigned)cdiv(n, 256), 256, 0, st>>>(scal, n, s.c, s.nwin, s.NB, s.counts, s.err);
+        k_digit_counts<C><<<(unsigned)cdiv(n, 256), 256, 0, st>>>(scal, n, s.c, s.nwin, ws, s.counts, s.err);
         launches++;
       }
       k_scan_reduce<<<(unsigned)s.ntiles, SCAN_THREADS, 0, st>>>(s.counts, s.F, s.tiles);
@@ -131,25 +183,29 @@ struct Ops final : CurveOps {
       k_scan_apply<<<(unsigned)s.ntiles, SCAN_THREADS, 0, st>>>(s.counts, s.F, s.tiles, s.goff, s.cursor);
       launches += 3;
       if (n) {
-        k_digit_scatter<C><<<(unsigned)cdiv(n, 256), 256, 0, st>>>(scal, n, s.c, s.nwin, s.NB, s.cursor, s.sorted);
+        k_digit_scatter<C><<<(unsigned)cdiv(n, 256), 256, 0, st>>>(scal, n, s.c, s.nwin, ws, istride, s.cursor, s.sorted);
         launches++;
       }
     }
     CK(cudaGetLastError());
     if (timed) CK(cudaEventRecord(s.ev[EV_SORT], st));
     // a4: accumulate + fixup
-    k_accumulate<C><<<(unsigned)cdiv(s.acc_threads, 128), 128, 0, st>>>(s.pts, s.sorted, s.goff, (uint32_t)s.F, s.slice,
-                                                                        s.buckets, s.carry_pts, s.carry_f, s.acc_threads);
+    k_accumulate<C><<<(unsigned)cdiv(s.acc_threads, 128), 128, 0, st>>>(pts, s.sorted, s.goff, (uint32_t)s.F,
+                                                                        s.buckets, s.carry_pts, s.carry_f, s.acc_threads,
+                                                                        s.nlong);
     launches++;
     CK(cudaGetLastError());
     if (timed) CK(cudaEventRecord(s.ev[EV_ACC], st));
-    k_fixup<C><<<(unsigned)cdiv(s.acc_threads, 128), 128, 0, st>>>(s.buckets, s.carry_pts, s.carry_f, s.acc_threads);
-    launches++;
+    k_fixup<C><<<(unsigned)cdiv(s.acc_threads, 128), 128, 0, st>>>(s.buckets, s.carry_pts, s.carry_f, s.acc_threads,
+                                                                   s.nlong, s.longs);
+    k_fixup_long<C><<<(unsigned)s.sms, FIX_THREADS, FIX_THREADS * XW_ * 4, st>>>(s.buckets, s.carry_pts, s.carry_f,
+                                                                                s.acc_threads, s.nlong, s.longs);
+    launches += 2;
     CK(cudaGetLastError());
     if (timed) CK(cudaEventRecord(s.ev[EV_FIX], st));
     // a5: bucket reduce
-    const uint32_t total = (uint32_t)s.nwin * s.nseg;
-    k_bucket_segments<C><<<(unsigned)cdiv(total, 128), 128, 0, st>>>(s.buckets, s.goff, s.nwin, s.NB, s.seg, s.nseg, s.segA);
+    const uint32_t total = (uint32_t)s.nset * s.nseg;
+    k_bucket_segments<C><<<(unsigned)cdiv(total, 128), 128, 0, st>>>(s.buckets, s.goff, s.nset, s.NB, s.seg, s.nseg, s.segA);
     launches++;
     uint32_t nin = s.nseg;
     uint32_t* src = s.segA;
@@ -158,17 +214,17 @@ struct Ops final : CurveOps {
       const uint32_t group = nin > 32 ? 32 : nin;
       const uint32_t nout = (uint32_t)cdiv(nin, group);
       uint32_t* out = nout == 1 ? s.W : dst;
-      k_sum_groups<C><<<(unsigned)cdiv((size_t)s.nwin * nout, 128), 128, 0, st>>>(src, nin, group, nout, s.nwin, out);
+      k_sum_groups<C><<<(unsigned)cdiv((size_t)s.nset * nout, 128), 128, 0, st>>>(src, nin, group, nout, s.nset, out);
       launches++;
       nin = nout;
       std::swap(src, dst);
       if (nout == 1) { src = s.W; break; }
     }
-    if (src != s.W) CK(cudaMemcpyAsync(s.W, src, (size_t)s.nwin * XW_ * 4, cudaMemcpyDeviceToDevice, st));
+    if (src != s.W) CK(cudaMemcpyAsync(s.W, src, (size_t)s.nset * XW_ * 4, cudaMemcpyDeviceToDevice, st));
     CK(cudaGetLastError());
     if (timed) CK(cudaEventRecord(s.ev[EV_RED], st));
     // a6: window combine
-    k_window_combine<C><<<1, 32, 0, st>>>(s.W, s.nwin, s.c, s.partial);
+    k_window_combine<C><<<1, 32, 0, st>>>(s.W, s.nset, s.c, s.partial);
     launches++;
     CK(cudaGetLastError());
     if (timed) CK(cudaEventRecord(s.ev[EV_COMB], st));

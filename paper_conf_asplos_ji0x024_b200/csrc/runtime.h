@@ -50,8 +50,10 @@ struct Shard {
   cudaEvent_t ev[EV_COUNT] = {};
   // configuration (depends on c)
   int c = 0, nwin = 0;
-  uint32_t NB = 0;     // buckets per window incl. bucket 0 = 2^(c-1) + 1
-  size_t F = 0;        // flat buckets = nwin * NB
+  int pre = 0;         // precomputed window table in use (f3): one bucket set for all windows
+  int nset = 0;        // bucket sets: nwin (pre = 0) or 1 (pre = 1)
+  uint32_t NB = 0;     // buckets per set incl. bucket 0 = 2^(c-1) + 1
+  size_t F = 0;        // flat buckets = nset * NB
   uint32_t acc_threads = 0, slice = 0;
   uint32_t seg = 0, nseg = 0;
   size_t ntiles = 0;
@@ -65,14 +67,23 @@ struct Shard {
            *W = nullptr, *partial = nullptr, *partials = nullptr, *tiles = nullptr, *err = nullptr,
            *result = nullptr;
   int32_t* carry_f = nullptr;
+  uint32_t* nlong = nullptr;   // k_fixup long-run list: count, and the runs' first carries
+  uint32_t* longs = nullptr;
+  int sms = 148;
   uint32_t *binCount = nullptr, *binOff = nullptr, *binCursor = nullptr, *binIdx = nullptr;
   uint16_t* binFine = nullptr;
   uint32_t* host_err = nullptr;  // pinned
+  // f3 precomputation: table[j][i] = 2^(j c) P_i, affine device form,
+  // [nwin][n][PW] words; built for window size table_c, kept across runs.
+  uint32_t* table = nullptr;
+  int table_c = 0;
+  float table_ms = 0;
 };
 
 struct Options {
   int c = 0, threads = 0, seg = 0;
   int sort = 0;  // 0: binned two-level sort (default), 1: direct global atomics (ablation)
+  int pre = 2;   // f3 precomputation: 0 off, 1 on, 2 auto (on when the table fits in memory)
 };
 
 // Per-curve kernels behind a virtual interface (one instance per curve, curve_*.cu).
@@ -84,8 +95,11 @@ struct CurveOps {
   virtual int PW() const = 0;
   virtual int XW() const = 0;
   virtual void points_to_mont(Shard& s, const uint32_t* in_dev, size_t n) = 0;
-  virtual void configure(const Options& o, Shard& s, int c) = 0;
+  // (re)allocates the scratch for window size c; pre = 1 uses (and if needed builds) the
+  // f3 precomputed table
+  virtual void configure(const Options& o, Shard& s, int c, int pre) = 0;
   virtual void free_scratch(Shard& s) = 0;
+  virtual void free_table(Shard& s) = 0;
   // enqueue a2..a6 on s.stream for the shard's scalars; the partial ends in s.partial.
   // Returns the number of kernels launched.
   virtual int enqueue_pipeline(Shard& s, const uint32_t* scal_dev, bool timed) = 0;
@@ -100,9 +114,11 @@ struct CurveOps {
 
 inline int num_windows(int lambda, int c) { return lambda / c + 1; }
 
-CurveOps* make_ops_bn254();
-CurveOps* make_ops_bls12_377();
-CurveOps* make_ops_bls12_381();
-CurveOps* make_ops_mnt4_753();
+// weak: a development build (tools/build.py --dev) may link a subset of the curve TUs;
+// a missing curve then reports MSM_ERR_CURVE.  The release build links all four.
+__attribute__((weak)) CurveOps* make_ops_bn254();
+__attribute__((weak)) CurveOps* make_ops_bls12_377();
+__attribute__((weak)) CurveOps* make_ops_bls12_381();
+__attribute__((weak)) CurveOps* make_ops_mnt4_753();
 
 }  // namespace msmrt

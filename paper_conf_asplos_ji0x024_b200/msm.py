@@ -24,8 +24,10 @@ OPT_WINDOW_BITS = 1
 OPT_ACC_THREADS = 2
 OPT_SEG_LEN = 3
 OPT_SORT = 4
+OPT_PRECOMPUTE = 5
 OPT_NWIN = 101
 OPT_NONEMPTY = 102
+OPT_NSETS = 103
 
 ERRORS = {
     0: "ok", -1: "invalid argument", -2: "unknown curve", -3: "CUDA error", -4: "device out of memory",
@@ -46,7 +48,7 @@ class Stats(ctypes.Structure):
         ("fixup_ms", ctypes.c_float), ("reduce_ms", ctypes.c_float), ("combine_ms", ctypes.c_float),
         ("finalize_ms", ctypes.c_float), ("total_ms", ctypes.c_float), ("window_bits", ctypes.c_int),
         ("nwin", ctypes.c_int), ("acc_threads", ctypes.c_int), ("acc_launches", ctypes.c_int),
-        ("entries", ctypes.c_uint64),
+        ("entries", ctypes.c_uint64), ("precompute", ctypes.c_int), ("table_ms", ctypes.c_float),
     ]
 
     def as_dict(self):
@@ -191,8 +193,9 @@ class Context:
         return out
 
     def windows(self, scalars, with_buckets=False):
-        """Debug: window sums W_j (and bucket sums B_{j,b}) as affine int pairs."""
-        nwin = self.get_option(OPT_NWIN)
+        """Debug: per-set sums W_s = sum_b b*B_{s,b} (and bucket sums B_{s,b}) as affine int
+        pairs.  Without the f3 table the sets are the windows j; with it there is one set."""
+        nwin = self.get_option(OPT_NSETS)
         c = self.get_option(OPT_WINDOW_BITS)
         W = np.zeros(nwin * 2 * self.L32, dtype=np.uint32)
         B = np.zeros(nwin * ((1 << (c - 1)) + 1) * 2 * self.L32, dtype=np.uint32) if with_buckets else None

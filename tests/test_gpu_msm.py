@@ -24,9 +24,11 @@ def closed(name, ks, es):
     return ec.to_output(omsm.msm_closed_form(ks, es, CURVES[name]))
 
 
-def run(lib, name, Ps, ks, c=None, ngpus=1):
+def run(lib, name, Ps, ks, c=None, ngpus=1, pre=None):
     ctx = lib.Context(name, points_to_words(Ps, name), ngpus=ngpus, n=len(Ps))
     try:
+        if pre is not None:
+            ctx.set_option(lib.OPT_PRECOMPUTE, pre)
         if c:
             ctx.set_option(lib.OPT_WINDOW_BITS, c)
         return ctx.run(synth.ints_to_words(ks, S_W[name]) if ks else np.zeros((0, S_W[name]), np.uint32))
@@ -99,7 +101,9 @@ def test_stage_parity_buckets_and_windows(lib, name):
     Ps, es, _, _ = progression(name, n, 24)
     ks = synth.words_to_ints(synth.scalars(c.r, n, 77))
     ctx = lib.Context(name, points_to_words(list(Ps), name), n=n)
+    ctx.set_option(lib.OPT_PRECOMPUTE, 0)
     ctx.set_option(1, cbits)
+    assert ctx.get_option(lib.OPT_NSETS) == ctx.get_option(lib.OPT_NWIN)
     Ws, Bs = ctx.windows(synth.ints_to_words(ks, S_W[name]), with_buckets=True)
     ctx.close()
     Bo = stages.bucket_sums(ks, list(Ps), cbits, c)
@@ -180,6 +184,7 @@ def test_sort_variants(lib, name, sort, cbits):
     Ps, es, _, _ = progression(name, n, 28)
     ks = synth.words_to_ints(synth.scalars(c.r, n, 40 + cbits))
     ctx = lib.Context(name, points_to_words(list(Ps), name), n=n)
+    ctx.set_option(lib.OPT_PRECOMPUTE, 0)
     ctx.set_option(lib.OPT_SORT, sort)
     ctx.set_option(lib.OPT_WINDOW_BITS, cbits)
     assert ctx.get_option(lib.OPT_SORT) == sort
@@ -205,4 +210,93 @@ def test_large_c_binned_sort(lib):
     for cbits in (20, 22):
         ctx.set_option(lib.OPT_WINDOW_BITS, cbits)
         assert ctx.run(synth.ints_to_words(ks, 8)) == closed(name, ks, es), cbits
+    ctx.close()
+
+
+@pytest.mark.parametrize("name", NAMES)
+def test_precompute_modes(lib, name):
+    """f3 table on / off / auto: same result (closed form) at several c,
+    ragged n, with O points and duplicates; the option reports the mode in use."""
+    c = CURVES[name]
+    n = 257 if name != "mnt4_753" else 65
+    Ps, es, _, _ = progression(name, n, 30)
+    Ps = list(Ps)
+    Ps[5] = None          # O in the table stays O
+    Ps[9] = Ps[8]         # duplicate point: doubling inside a shared bucket
+    ks = synth.words_to_ints(synth.scalars(c.r, n, 51))
+    ks[8], ks[9] = ks[9], ks[9]
+    e = [0 if P is None else x for P, x in zip(Ps, es)]
+    e[9] = es[8]
+    want = closed(name, ks, e)
+    ctx = lib.Context(name, points_to_words(Ps, name), n=n)
+    sw = synth.ints_to_words(ks, S_W[name])
+    for pre in (1, 0, 2):
+        ctx.set_option(lib.OPT_PRECOMPUTE, pre)
+        for cbits in ((3, 8, 13) if name != "mnt4_753" else (6, 11)):
+            ctx.set_option(lib.OPT_WINDOW_BITS, cbits)
+            assert ctx.run(sw) == want, (pre, cbits)
+            if pre != 2:
+                assert ctx.get_option(lib.OPT_PRECOMPUTE) == pre
+                assert ctx.get_option(lib.OPT_NSETS) == (1 if pre else ctx.get_option(lib.OPT_NWIN))
+        ctx.set_option(lib.OPT_WINDOW_BITS, 0)
+        assert ctx.run(sw) == want, (pre, "auto c")
+    assert ctx.stats()["precompute"] in (0, 1)
+    ctx.close()
+
+
+@pytest.mark.parametrize("name", ["bn254", "bls12_377", "mnt4_753"])
+def test_stage_parity_precomputed(lib, name):
+    """With the f3 table: every bucket sum of the single shared set equals the oracle's
+    B^pre_b = sum over (i, j) of sgn(d_ij) 2^(jc) P_i, and its reduce is the MSM."""
+    c = CURVES[name]
+    n = 90 if name != "mnt4_753" else 30
+    cbits = 6 if name != "mnt4_753" else 9
+    Ps, es, _, _ = progression(name, n, 31)
+    ks = synth.words_to_ints(synth.scalars(c.r, n, 78))
+    ctx = lib.Context(name, points_to_words(list(Ps), name), n=n)
+    ctx.set_option(lib.OPT_PRECOMPUTE, 1)
+    ctx.set_option(lib.OPT_WINDOW_BITS, cbits)
+    assert ctx.get_option(lib.OPT_NSETS) == 1
+    Ws, Bs = ctx.windows(synth.ints_to_words(ks, S_W[name]), with_buckets=True)
+    ctx.close()
+    Bo = stages.bucket_sums_precomputed(ks, list(Ps), cbits, c)
+    for b in range(1, len(Bo)):
+        assert Bs[0][b] == ec.to_output(Bo[b]), b
+    assert Ws == [closed(name, ks, es)]
+
+
+@pytest.mark.parametrize("name", ["bn254", "bls12_381"])
+@pytest.mark.parametrize("kind", ["ones", "equal", "skewed"])
+def test_fixup_long_runs(lib, name, kind):
+    """Heavy buckets spanning many accumulation slices (skewed scalars, many threads):
+    k_fixup hands runs of > 8 carries to k_fixup_long's block tree."""
+    c = CURVES[name]
+    n = 3000
+    Ps, es, _, _ = progression(name, n, 32)
+    ks = synth.words_to_ints(synth.pattern_scalars(c.r, n, 6, kind))
+    want = closed(name, ks, es)
+    ctx = lib.Context(name, points_to_words(list(Ps), name), n=n)
+    sw = synth.ints_to_words(ks, S_W[name])
+    for pre in (0, 1):
+        ctx.set_option(lib.OPT_PRECOMPUTE, pre)
+        ctx.set_option(lib.OPT_WINDOW_BITS, 8)
+        for threads in (1, 37, 4096, 20000):
+            ctx.set_option(lib.OPT_ACC_THREADS, threads)
+            assert ctx.run(sw) == want, (pre, threads)
+    ctx.close()
+
+
+@pytest.mark.parametrize("cbits", [15, 17])
+def test_degenerate_top_window(lib, cbits):
+    """c dividing 255: the top window holds only the carry digit (bucket 1 gets ~n/2
+    entries) -- correct and not serialised in k_fixup."""
+    name = "bls12_381"
+    c = CURVES[name]
+    n = 4000
+    Ps, es, _, _ = progression(name, n, 33)
+    ks = synth.words_to_ints(synth.scalars(c.r, n, 61))
+    ctx = lib.Context(name, points_to_words(list(Ps), name), n=n)
+    ctx.set_option(lib.OPT_PRECOMPUTE, 0)
+    ctx.set_option(lib.OPT_WINDOW_BITS, cbits)
+    assert ctx.run(synth.ints_to_words(ks, 8)) == closed(name, ks, es)
     ctx.close()

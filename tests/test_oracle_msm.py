@@ -89,3 +89,30 @@ def test_synth_scalars_in_range():
         ks = synth.words_to_ints(synth.scalars(c.r, 500, 1))
         assert all(0 <= k < c.r for k in ks)
         assert max(ks).bit_length() >= c.lam - 3
+
+
+@pytest.mark.parametrize("c", ALL, ids=lambda c: c.name)
+def test_precomputed_route(c):
+    """f3: the table rows are 2^(jc) P (checked with the library-style
+    double-and-add ec.mul), the shared bucket set is sum_j 2^(jc) B_{j,b} of the per-window
+    model, and its single bucket-reduce is the MSM (closed form)."""
+    n = 6 if c.name == "mnt4_753" else 14
+    e0, d = synth.point_seeds(c.r, 8)
+    Ps = points.progression_points(e0, d, n, c)
+    es = points.progression_scalars(e0, d, n, c)
+    ks = synth.words_to_ints(synth.scalars(c.r, n, 123))
+    ks[0], ks[1] = c.r - 1, 0
+    want = msm.msm_closed_form(ks, es, c)
+    big = c.name == "mnt4_753"
+    for cc in ((5, 9) if not big else (16,)):
+        T = stages.precomputed_table(Ps[:2], cc, c)
+        for j in (range(len(T)) if not big else (1, 2, len(T) - 1)):
+            assert T[j][1] == ec.mul(pow(2, j * cc), Ps[1], c)
+        Bp = stages.bucket_sums_precomputed(ks, Ps, cc, c)
+        Bw = stages.bucket_sums(ks, Ps, cc, c)
+        for b in (range(1, len(Bp)) if not big else ()):
+            acc = None
+            for j in range(len(Bw)):
+                acc = ec.add(acc, ec.mul(pow(2, j * cc), Bw[j][b], c) if Bw[j][b] else None, c)
+            assert Bp[b] == acc, b
+        assert stages.msm_precomputed(ks, Ps, cc, c) == want

@@ -42,11 +42,25 @@ def compile_one(src, force, build_dir=BUILD, defines=()):
     return obj, "built"
 
 
-def build(jobs=8, force=False, verbose=True, only=None, defines=(), out=OUT, build_dir=BUILD):
+def build(jobs=8, force=False, verbose=True, only=None, defines=(), out=OUT, build_dir=BUILD, dev=None):
     """only: curve TU names to (re)compile (others reuse build_dir objects: dev/variants);
-    defines: extra -D macros (kernel variants for A/B runs)."""
+    defines: extra -D macros (kernel variants for A/B runs);
+    dev: curve TU names to compile AND link (with engine.cu) -- a fast development library
+    in which the other curves report MSM_ERR_CURVE (their factories are weak symbols)."""
     os.makedirs(build_dir, exist_ok=True)
     srcs = sorted(glob.glob(os.path.join(CSRC, "*.cu")))
+    if dev:
+        srcs = [s for s in srcs if "curve_" not in s or any(d in s for d in dev)]
+        res = [compile_one(s, force, build_dir, defines) for s in srcs] if jobs == 1 else \
+            list(cf.ThreadPoolExecutor(max_workers=jobs).map(lambda s: compile_one(s, force, build_dir, defines), srcs))
+        objs = [o for o, _ in res]
+        cmd = [NVCC, "-gencode", "arch=compute_100a,code=sm_100a", "-shared", "-o", out] + objs
+        r = subprocess.run(cmd, capture_output=True, text=True)
+        if r.returncode != 0:
+            raise RuntimeError("link failed:\n" + r.stderr[-4000:])
+        if verbose:
+            print("built (dev: %s)" % ",".join(dev), out)
+        return out
     if only:
         keep = [s for s in srcs if "curve_" not in s or any(o in s for o in only)]
         stale = [s for s in srcs if s not in keep]
@@ -83,9 +97,11 @@ if __name__ == "__main__":
     ap.add_argument("-D", action="append", default=[], help="extra macro for a variant build")
     ap.add_argument("--out", default=OUT)
     ap.add_argument("--build-dir", default=BUILD)
+    ap.add_argument("--dev", default="", help="comma-separated curve TUs: compile+link only these (fast dev lib)")
     a = ap.parse_args()
     try:
-        build(a.j, a.force, only=[o for o in a.only.split(",") if o], defines=a.D, out=a.out, build_dir=a.build_dir)
+        build(a.j, a.force, only=[o for o in a.only.split(",") if o], defines=a.D, out=a.out, build_dir=a.build_dir,
+              dev=[d for d in a.dev.split(",") if d] or None)
     except RuntimeError as e:
         print(e, file=sys.stderr)
         sys.exit(1)
