@@ -60,7 +60,9 @@ enum {
   MSM_OPT_WINDOW_BITS = 1,    /* c in [2, 24]; 0 = automatic (cost model). Reallocates scratch. */
   MSM_OPT_ACC_THREADS = 2,    /* accumulation threads per device; 0 = automatic            */
   MSM_OPT_SEG_LEN = 3,        /* buckets per bucket-reduce segment; 0 = automatic          */
-  MSM_OPT_SORT = 4,           /* a3 variant: 0 = two-level binned sort (default), 1 = direct global atomics */
+  MSM_OPT_SORT = 4,           /* a3 variant: 0 = auto (default: 3 for >= 2^21 entries, else 2),
+                                 1 = direct global atomics (ablation), 2 = two-level binned,
+                                 3 = three-level staged (coalesced runs); get returns 1..3   */
   MSM_OPT_PRECOMPUTE = 5,     /* f3 window table 2^(jc) P_i: 0 off, 1 on,
                                  2 auto (default: on when the table fits in device memory).
                                  With it all windows share one bucket set; building the table

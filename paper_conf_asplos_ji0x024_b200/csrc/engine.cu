@@ -66,7 +66,7 @@ size_t scratch_bytes(size_t n, int lambda, int c, int XW, bool pre) {
   const size_t nwin = num_windows(lambda, c);
   const size_t sets = pre ? 1 : nwin;
   const size_t NB = ((size_t)1 << (c - 1)) + 1;
-  return n * nwin * 10 + sets * NB * ((size_t)XW * 4 + 12) + ((size_t)1 << 28);
+  return n * nwin * 22 + sets * NB * ((size_t)XW * 4 + 12) + ((size_t)1 << 28);
 }
 
 // Chooses (c, pre) for one shard: opt.c / opt.pre when fixed; otherwise the cheapest
@@ -471,7 +471,7 @@ int msm_set_option(msm_context* ctx, int key, long value) {
       ctx->opt.seg = (int)value;
       break;
     case MSM_OPT_SORT:
-      if (value < 0 || value > 1) return MSM_ERR_ARG;
+      if (value < 0 || value > 3) return MSM_ERR_ARG;
       ctx->opt.sort = (int)value;
       break;
     case MSM_OPT_PRECOMPUTE:

@@ -57,17 +57,38 @@ struct Fp {
 // two chains that start from 0 — independent of every earlier column — and the carry is
 // added afterwards, so a lone warp overlaps the columns instead of walking one long
 // dependency chain (2 extra ALU ops per column, irrelevant off the throughput path).
-template <class C, bool SQR, bool LAT, int K, bool PREV_SPLIT>
-DEVI void fmul_col(uint32_t* r, const uint32_t* a, const uint32_t* b, const uint32_t* a2, uint32_t* m, u64 cA, u64 cM) {
+// Shape of product-scan column K: a*b terms i in [lo, hiA], m*p terms i in [lo, hiM] plus
+// m_K p_0 (K < L).  A 64-bit accumulator holds MAXT products of W-bit limbs plus a carry;
+// a column with more terms splits a*b and m*p over two accumulators ("split").
+template <class C>
+__host__ __device__ constexpr bool col_single(int K) {
+  const int L = C::L, W = C::W;
+  const int MAXT = (W == 30) ? 15 : (W == 29 ? 63 : 255);
+  const int lo = K - L + 1 > 0 ? K - L + 1 : 0;
+  const int hiA = K < L - 1 ? K : L - 1;
+  const int hiM = (K - 1) < (L - 1) ? K - 1 : L - 1;
+  const int nA = hiA - lo + 1;
+  const int nM = (hiM >= lo ? hiM - lo + 1 : 0) + (K < L ? 1 : 0);
+  return (C::NACC == 1) || (nA + nM <= MAXT);
+}
+
+template <class C, int K>
+struct ColShape {
+  static constexpr int L = C::L;
+  static constexpr int lo = K - L + 1 > 0 ? K - L + 1 : 0;
+  static constexpr int hiA = K < L - 1 ? K : L - 1;
+  static constexpr int hiM = (K - 1) < (L - 1) ? K - 1 : L - 1;
+  static constexpr bool single = col_single<C>(K);
+  static constexpr bool prev_split = K > 0 && !col_single<C>(K - 1);
+};
+
+template <class C, bool SQR, bool LAT, int K>
+DEVI void fmul_step(uint32_t* r, const uint32_t* a, const uint32_t* b, const uint32_t* a2, uint32_t* m, u64& cA, u64& cM) {
+  using S = ColShape<C, K>;
   constexpr int L = C::L, W = C::W;
   constexpr uint32_t MASK = (1u << W) - 1;
-  constexpr int MAXT = (W == 30) ? 15 : (W == 29 ? 63 : 255);
-  constexpr int lo = K - L + 1 > 0 ? K - L + 1 : 0;
-  constexpr int hiA = K < L - 1 ? K : L - 1;
-  constexpr int hiM = (K - 1) < (L - 1) ? K - 1 : L - 1;
-  constexpr int nA = hiA - lo + 1;
-  constexpr int nM = (hiM >= lo ? hiM - lo + 1 : 0) + (K < L ? 1 : 0);
-  constexpr bool single = (C::NACC == 1) || (nA + nM <= MAXT);
+  constexpr int lo = S::lo, hiA = S::hiA, hiM = S::hiM;
+  constexpr bool single = S::single, PREV_SPLIT = S::prev_split;
   u64 accA;
   if constexpr (LAT) {
     u64 e0 = 0, e1 = 0;
@@ -128,11 +149,32 @@ DEVI void fmul_col(uint32_t* r, const uint32_t* a, const uint32_t* b, const uint
       nM_carry = (accM >> W) + (s >> W);
     }
   }
-  if constexpr (K + 1 < 2 * L - 1) {
-    fmul_col<C, SQR, LAT, K + 1, !single>(r, a, b, a2, m, nA_carry, nM_carry);
-  } else {
-    r[L - 1] = (uint32_t)(single ? nA_carry : nA_carry + nM_carry);
-  }
+  if constexpr (K == 2 * L - 2) r[L - 1] = (uint32_t)(single ? nA_carry : nA_carry + nM_carry);
+  cA = nA_carry;
+  cM = nM_carry;
+}
+
+// One column per template instance: every index is a compile-time constant, so the whole
+// product scan is straight-line code on registers (no reliance on the loop unroller, which
+// gives up on 25 large column bodies and then spills m[] to local memory).
+template <class C, bool SQR, bool LAT, int K>
+DEVI void fmul_cols(uint32_t* r, const uint32_t* a, const uint32_t* b, const uint32_t* a2, uint32_t* m, u64 cA, u64 cM) {
+  fmul_step<C, SQR, LAT, K>(r, a, b, a2, m, cA, cM);
+  if constexpr (K + 1 < 2 * C::L - 1) fmul_cols<C, SQR, LAT, K + 1>(r, a, b, a2, m, cA, cM);
+}
+
+// Two independent products column-interleaved: four accumulation chains instead of two,
+// so the IMAD.WIDE latency of one product's column hides behind the other's (ILP without
+// more warps; the accumulation kernel runs at 2 warps per scheduler).  r1 / r2 may alias
+// their OWN inputs only (as for fmul), never the other product's inputs.
+template <class C, bool SQR, int K>
+DEVI void fmul2_cols(uint32_t* r1, const uint32_t* a1, const uint32_t* b1, const uint32_t* a21, uint32_t* m1,
+                     u64 cA1, u64 cM1, uint32_t* r2, const uint32_t* a2, const uint32_t* b2, const uint32_t* a22,
+                     uint32_t* m2, u64 cA2, u64 cM2) {
+  fmul_step<C, SQR, false, K>(r1, a1, b1, a21, m1, cA1, cM1);
+  fmul_step<C, SQR, false, K>(r2, a2, b2, a22, m2, cA2, cM2);
+  if constexpr (K + 1 < 2 * C::L - 1)
+    fmul2_cols<C, SQR, K + 1>(r1, a1, b1, a21, m1, cA1, cM1, r2, a2, b2, a22, m2, cA2, cM2);
 }
 
 template <class C, bool SQR, bool LAT = false>
@@ -144,7 +186,19 @@ DEVI void fmul_impl(uint32_t* r, const uint32_t* a, const uint32_t* b) {
 #pragma unroll
     for (int i = 0; i < L; i++) a2[i] = a[i] << 1;
   }
-  fmul_col<C, SQR, LAT, 0, false>(r, a, b, a2, m, 0ull, 0ull);
+  fmul_cols<C, SQR, LAT, 0>(r, a, b, a2, m, 0ull, 0ull);
+}
+
+// r1 = a1*b1, r2 = a2*b2 (SQR: r1 = a1^2, r2 = a2^2), same contract as fmul
+template <class C, bool SQR = false>
+DEVI void fmul2(uint32_t* r1, const uint32_t* a1, const uint32_t* b1, uint32_t* r2, const uint32_t* a2, const uint32_t* b2) {
+  constexpr int L = C::L;
+  uint32_t m1[L], m2[L], d1[L], d2[L];
+  if constexpr (SQR) {
+#pragma unroll
+    for (int i = 0; i < L; i++) { d1[i] = a1[i] << 1; d2[i] = a2[i] << 1; }
+  }
+  fmul2_cols<C, SQR, 0>(r1, a1, b1, d1, m1, 0ull, 0ull, r2, a2, b2, d2, m2, 0ull, 0ull);
 }
 
 template <class C>

@@ -541,6 +541,9 @@ __global__ void __launch_bounds__(BIN_THREADS) k_bin_scatter(const uint32_t* __r
 // k_bin_sort_impl (one block per flat bin, nfine = 2^shift <= 8192) is defined with the
 // scan helpers above.
 
+#include "sort3.cuh"
+
+
 // ---------------------------------------------------------------------------------------
 // number of non-empty flat buckets (statistics only)
 static __global__ void k_count_nonempty(const uint32_t* __restrict__ goff, size_t F, unsigned long long* out) {
@@ -564,6 +567,21 @@ DEVI bool point_for_entry(uint32_t* x, uint32_t* y, const uint32_t* __restrict__
   if (fis_zero<C, 2>(y)) return false;
   if (e & SIGN_BIT) fneg<C, 2>(y, y);
   return true;
+}
+
+#ifndef MSM_ACC_PREFETCH
+#define MSM_ACC_PREFETCH 1
+#endif
+#ifndef MSM_ACC_DUAL
+#define MSM_ACC_DUAL 1  // k_accumulate: column-interleaved multiplication pairs (xyzz_acc_hot)
+#endif
+
+// L1 prefetch of the (at most two) 128-B lines holding the stored point of entry e
+template <class C>
+DEVI void prefetch_point(const uint32_t* __restrict__ pts, uint32_t e) {
+  const char* a = reinterpret_cast<const char*>(pts + (size_t)(e & ~SIGN_BIT) * Layout<C>::PW);
+  asm volatile("prefetch.global.L1 [%0];" ::"l"(a));
+  asm volatile("prefetch.global.L1 [%0];" ::"l"(a + Layout<C>::PW * 4 - 4));
 }
 
 template <class C>
@@ -607,8 +625,22 @@ __global__ void __launch_bounds__(128, MSM_ACC_MINB) k_accumulate(const uint32_t
   bool ok = point_for_entry<C>(x, y, pts, __ldg(sorted + e0));
   acc_start<C>(acc, x, y, ok);
   int32_t my_carry = -1;
+#if MSM_ACC_PREFETCH
+  // the gathered point of entry e+1 is prefetched into L1 one PACC ahead (its index
+  // read two ahead), so the random 8L-byte gather does not stall the next iteration
+  uint32_t ent1 = e0 + 1 < e1 ? __ldg(sorted + e0 + 1) : 0u;
+  uint32_t ent2 = e0 + 2 < e1 ? __ldg(sorted + e0 + 2) : 0u;
+  if (e0 + 1 < e1) prefetch_point<C>(pts, ent1);
+#endif
   for (uint32_t e = e0 + 1; e < e1; e++) {
+#if MSM_ACC_PREFETCH
+    const uint32_t ent = ent1;
+    ent1 = ent2;
+    if (e + 1 < e1) prefetch_point<C>(pts, ent1);
+    if (e + 2 < e1) ent2 = __ldg(sorted + e + 2);
+#else
     const uint32_t ent = __ldg(sorted + e);
+#endif
     ok = point_for_entry<C>(x, y, pts, ent);
     if (e == end) {
       if (head) { store_xyzz<C>(carry_pts + (size_t)t * XW, acc); my_carry = (int32_t)f; head = false; }
@@ -616,7 +648,14 @@ __global__ void __launch_bounds__(128, MSM_ACC_MINB) k_accumulate(const uint32_t
       do { f++; end = __ldg(goff + f + 1); } while (end <= e);
       acc_start<C>(acc, x, y, ok);
     } else if (ok) {
+#if MSM_ACC_DUAL
+      if (xyzz_acc_hot<C>(acc, x, y)) {  // rare: the point equals the accumulator
+        Xyzz<C> T = acc;
+        xyzz_dbl<C>(acc, T);
+      }
+#else
       xyzz_acc<C>(acc, x, y);
+#endif
     }
   }
   if (head) { store_xyzz<C>(carry_pts + (size_t)t * XW, acc); my_carry = (int32_t)f; }

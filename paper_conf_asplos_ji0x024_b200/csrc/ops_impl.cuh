@@ -32,6 +32,9 @@ struct Ops final : CurveOps {
     dfree(s.carry_pts); dfree(s.carry_f); dfree(s.segA); dfree(s.segB); dfree(s.W); dfree(s.tiles);
     dfree(s.binCount); dfree(s.binOff); dfree(s.binCursor); dfree(s.binIdx); dfree(s.binFine);
     dfree(s.nlong); dfree(s.longs);
+    dfree(s.s3Count); dfree(s.s3Off); dfree(s.s3Cursor); dfree(s.s3Sub);
+    dfree(s.s3SubCount); dfree(s.s3SubCursor); dfree(s.s3Tiles);
+    dfree(s.s3k1); dfree(s.s3v1); dfree(s.s3k2); dfree(s.s3v2);
   }
 
   void free_table(Shard& s) override {
@@ -82,7 +85,10 @@ struct Ops final : CurveOps {
     s.NB = (1u << (c - 1)) + 1;
     s.F = (size_t)s.nset * s.NB;
     s.ntiles = cdiv(s.F, SCAN_TILE);
-    s.sort_mode = o.sort;
+    // a3 variant: the staged three-level sort for large entry counts, the binned two-level
+    // sort below ~2^21 entries (fewer launches)
+    const size_t Mmax0 = s.n * (size_t)s.nwin;
+    s.sort_mode = o.sort ? o.sort : (Mmax0 >= ((size_t)1 << 21) ? 3 : 2);
     s.shift = 0;
     while (s.shift < 13 && (size_t)s.nset * ((((size_t)1 << (c - 1)) >> s.shift) + 1) > 13000) s.shift++;
     s.nbin = (uint32_t)((((size_t)1 << (c - 1)) >> s.shift) + 1);
@@ -131,8 +137,37 @@ struct Ops final : CurveOps {
     dalloc(&s.segA, (size_t)s.nset * s.nseg * XW_);
     dalloc(&s.segB, (size_t)s.nset * cdiv(s.nseg, 32) * XW_);
     dalloc(&s.W, (size_t)s.nset * XW_);
-    dalloc(&s.tiles, std::max(s.ntiles, s.ntiles_bin) + 1);
-    if (s.sort_mode == 0) {
+    dalloc(&s.tiles, std::max(std::max(s.ntiles, s.ntiles_bin), cdiv((size_t)1 << 18, SCAN_TILE)) + 1);
+    if (s.sort_mode == 3) {
+      // key bits: b3 resolved per sub-bin in shared memory (~8K entries per sub-bin),
+      // b1, b2 <= 9 per partition pass
+      int KB = 1;
+      while (((size_t)1 << KB) < s.F) KB++;
+      int b3 = (int)std::lround(std::log2(8192.0 * (double)s.F / (double)std::max<size_t>(Mmax, 1)));
+      b3 = std::max(1, std::min(b3, 12));
+      b3 = std::min(b3, KB);
+      if (KB - b3 > 18) b3 = KB - 18;
+      const int rest = KB - b3;
+      s.s3_b2 = std::min(9, rest / 2);
+      s.s3_b1 = rest - s.s3_b2;
+      s.s3_b3 = b3;
+      const size_t NC1 = (size_t)1 << s.s3_b1, NC2 = (size_t)1 << s.s3_b2;
+      dalloc(&s.s3Count, NC1);
+      dalloc(&s.s3Off, NC1 + 1);
+      dalloc(&s.s3Cursor, NC1);
+      dalloc(&s.s3Sub, NC1 * NC2 + 1);
+      dalloc(&s.s3SubCount, NC1 * NC2);
+      dalloc(&s.s3SubCursor, NC1 * NC2);
+      dalloc(&s.s3Tiles, NC1 + 1);
+      dalloc(&s.s3k1, Mmax);
+      dalloc(&s.s3v1, Mmax);
+      dalloc(&s.s3k2, Mmax);
+      dalloc(&s.s3v2, Mmax);
+      CK(cudaFuncSetAttribute(k_s3_part1<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * S3_TILE * 4));
+      CK(cudaFuncSetAttribute(k_s3_part2, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * S3_TILE * 4));
+      CK(cudaFuncSetAttribute(k_s3_part3, cudaFuncAttributeMaxDynamicSharedMemorySize, (S3_CAP + S3_MAXFINE) * 4));
+    }
+    if (s.sort_mode == 2) {
       dalloc(&s.binCount, s.FB);
       dalloc(&s.binOff, s.FB + 1);
       dalloc(&s.binCursor, s.FB);
@@ -150,7 +185,41 @@ struct Ops final : CurveOps {
     const uint32_t* pts = s.pre ? s.table : s.pts;
     if (timed) CK(cudaEventRecord(s.ev[EV_H2D], st));
     // a2 + a3: digits, histogram, scan, scatter
-    if (s.sort_mode == 0) {
+    if (s.sort_mode == 3) {
+      const uint32_t NC1 = 1u << s.s3_b1, NC2 = 1u << s.s3_b2;
+      const int sh1 = s.s3_b2 + s.s3_b3;
+      CK(cudaMemsetAsync(s.s3Count, 0, NC1 * sizeof(uint32_t), st));
+      if (n) {
+        k_s3_count1<C><<<(unsigned)cdiv(n, S3_THREADS * 16), S3_THREADS, 0, st>>>(scal, n, s.c, s.nwin, ws, sh1, NC1,
+                                                                               s.s3Count, s.err);
+        launches++;
+      }
+      const size_t nt = cdiv(NC1, SCAN_TILE);
+      k_scan_reduce<<<(unsigned)nt, SCAN_THREADS, 0, st>>>(s.s3Count, NC1, s.tiles);
+      k_scan_tiles<<<1, 1024, 0, st>>>(s.tiles, nt, s.s3Off + NC1);
+      k_scan_apply<<<(unsigned)nt, SCAN_THREADS, 0, st>>>(s.s3Count, NC1, s.tiles, s.s3Off, s.s3Cursor);
+      launches += 3;
+      const uint32_t tp = (uint32_t)std::max(1, S3_TILE / s.nwin);
+      if (n) {
+        k_s3_part1<C><<<(unsigned)cdiv(n, tp), S3_THREADS, 2 * S3_TILE * 4, st>>>(scal, n, s.c, s.nwin, ws, istride, sh1,
+                                                                                NC1, tp, s.s3Cursor, s.s3k1, s.s3v1);
+        launches++;
+      }
+      const unsigned maxTiles = (unsigned)(cdiv(std::max<size_t>(s.n * (size_t)s.nwin, 1), S3_TILE) + NC1);
+      const size_t nsub = (size_t)NC1 * NC2, nts = cdiv(nsub, SCAN_TILE);
+      k_s3_tiles<<<1, S3_THREADS, 0, st>>>(s.s3Off, NC1, s.s3Tiles);
+      CK(cudaMemsetAsync(s.s3SubCount, 0, nsub * sizeof(uint32_t), st));
+      k_s3_count2<<<maxTiles, S3_THREADS, 0, st>>>(s.s3Tiles, s.s3Off, NC1, s.s3_b3, NC2, s.s3k1, s.s3SubCount);
+      k_scan_reduce<<<(unsigned)nts, SCAN_THREADS, 0, st>>>(s.s3SubCount, nsub, s.tiles);
+      k_scan_tiles<<<1, 1024, 0, st>>>(s.tiles, nts, s.s3Sub + nsub);
+      k_scan_apply<<<(unsigned)nts, SCAN_THREADS, 0, st>>>(s.s3SubCount, nsub, s.tiles, s.s3Sub, s.s3SubCursor);
+      k_s3_part2<<<maxTiles, S3_THREADS, 2 * S3_TILE * 4, st>>>(s.s3Tiles, s.s3Off, NC1, s.s3_b3, NC2, s.s3k1, s.s3v1,
+                                                                s.s3SubCursor, s.s3k2, s.s3v2);
+      CK(cudaMemcpyAsync(s.goff + s.F, s.s3Off + NC1, 4, cudaMemcpyDeviceToDevice, st));
+      k_s3_part3<<<(unsigned)nsub, 256, (S3_CAP + (1u << s.s3_b3)) * 4, st>>>(s.s3Sub, s.s3_b3, (uint32_t)s.F, s.s3k2,
+                                                                             s.s3v2, s.goff, s.sorted);
+      launches += 7;
+    } else if (s.sort_mode == 2) {
       CK(cudaMemsetAsync(s.binCount, 0, s.FB * sizeof(uint32_t), st));
       const unsigned tiles = (unsigned)cdiv(std::max<size_t>(n, 1), BIN_TILE);
       if (n) {

@@ -58,7 +58,7 @@ struct Shard {
   uint32_t seg = 0, nseg = 0;
   size_t ntiles = 0;
   // binned sort geometry (a3): flat bins fb = j*nbin + (b >> shift), FB = nwin*nbin
-  int sort_mode = 0, shift = 0;
+  int sort_mode = 0, shift = 0;  // effective a3 variant (1, 2 or 3)
   uint32_t nbin = 0, FB = 0;
   size_t ntiles_bin = 0;
   // device buffers
@@ -72,6 +72,11 @@ struct Shard {
   int sms = 148;
   uint32_t *binCount = nullptr, *binOff = nullptr, *binCursor = nullptr, *binIdx = nullptr;
   uint16_t* binFine = nullptr;
+  // three-level staged sort (sort3.cuh): key bits b1 + b2 + b3 >= bits(F - 1)
+  int s3_b1 = 0, s3_b2 = 0, s3_b3 = 0;
+  uint32_t *s3Count = nullptr, *s3Off = nullptr, *s3Cursor = nullptr, *s3Sub = nullptr,
+           *s3k1 = nullptr, *s3v1 = nullptr, *s3k2 = nullptr, *s3v2 = nullptr, *s3SubCount = nullptr,
+           *s3SubCursor = nullptr, *s3Tiles = nullptr;
   uint32_t* host_err = nullptr;  // pinned
   // f3 precomputation: table[j][i] = 2^(j c) P_i, affine device form,
   // [nwin][n][PW] words; built for window size table_c, kept across runs.
@@ -82,7 +87,8 @@ struct Shard {
 
 struct Options {
   int c = 0, threads = 0, seg = 0;
-  int sort = 0;  // 0: binned two-level sort (default), 1: direct global atomics (ablation)
+  int sort = 0;  // a3 variant: 0 auto, 1 direct global atomics (ablation), 2 two-level binned,
+                 // 3 three-level staged (sort3.cuh)
   int pre = 2;   // f3 precomputation: 0 off, 1 on, 2 auto (on when the table fits in memory)
 };
 

@@ -1,0 +1,243 @@
+// a3, three-level staged counting sort (§3.2.1, Alg. 3).
+// Included inside namespace msmk by msm_kernels.cuh.
+//
+// The paper's bucket scatter ranks points per bucket in shared memory and reserves one
+// global range per (block, bucket) with one atomic (Alg. 3 lines 12-15), which
+// stops at s = 14 on A100 shared memory.  With c up to 24 a bucket set has up to
+// 2^23 buckets, so on B200 the scatter is split into three passes over a flat key
+// f = j*ws + b (the entry's flat bucket), each pass writing only long coalesced runs:
+//   P1  k_s3_part1   scalars -> (key, value) partitioned by the top b1 key bits: per tile
+//                    of E_T entries, shared-memory ranks, one global atomic per (tile, bin),
+//                    entries staged in shared memory in bin order and written as runs;
+//   P2  k_s3_count2 + scan + k_s3_part2: the P1 output, in tiles that never straddle a
+//                    P1 bin, partitioned by the next b2 bits the same way (sub-bin starts
+//                    from a global scan of the per-(bin, sub-bin) counts);
+//   P3  k_s3_part3   one block per sub-bin (2^b3 buckets, ~4-8K entries): a complete
+//                    counting sort in shared memory, written contiguously, plus goff.
+// The (i, j) entry value is (i + j*istride) | sign<<31 as in the other sort variants.
+// Why: the two-level binned sort (k_bin_scatter) wrote 6-B entries at random positions
+// of 8K bins; ncu measured 28.7 GB DRAM writes for 4.4 GB of entries at 2^26 (partial
+// sectors evicted before they fill) -- 31 ms of a 40 ms sort.
+
+constexpr int S3_THREADS = 512;
+constexpr int S3_TILE = 12288;       // staged entries per tile (96 KB of keys + values)
+constexpr int S3_CAP = 12288;        // largest sub-bin P3 sorts in shared memory
+constexpr int S3_MAXB = 512;         // max bins per partition pass (b1, b2 <= 9)
+constexpr int S3_MAXFINE = 4096;     // max buckets per sub-bin (b3 <= 12)
+
+// exclusive scan of cnt[0..N) in place (N <= blockDim.x * per-thread chunk); returns total
+__device__ __forceinline__ uint32_t s3_block_scan(uint32_t* cnt, uint32_t N, uint32_t* warp_sums) {
+  const uint32_t per = (N + blockDim.x - 1) / blockDim.x;
+  const uint32_t c0 = min(threadIdx.x * per, N), c1 = min(c0 + per, N);
+  uint32_t sum = 0;
+  for (uint32_t i = c0; i < c1; i++) sum += cnt[i];
+  uint32_t total;
+  uint32_t run = block_exclusive_scan(sum, warp_sums, &total);
+  for (uint32_t i = c0; i < c1; i++) {
+    const uint32_t v = cnt[i];
+    cnt[i] = run;
+    run += v;
+  }
+  __syncthreads();
+  return total;
+}
+
+// P1 histogram: binCount[f >> sh1] over all digits (tiles of BIN_TILE points); err |= 4
+// for k >= r
+template <class C>
+__global__ void __launch_bounds__(S3_THREADS) k_s3_count1(const uint32_t* __restrict__ scal, size_t n, int c, int nwin,
+                                                          uint32_t ws, int sh1, uint32_t NC1,
+                                                          uint32_t* __restrict__ binCount, uint32_t* err) {
+  __shared__ uint32_t hist[S3_MAXB];
+  for (uint32_t i = threadIdx.x; i < NC1; i += blockDim.x) hist[i] = 0;
+  __syncthreads();
+  const size_t base = (size_t)blockIdx.x * (S3_THREADS * 16);
+  bool bad = false;
+  for (int q = 0; q < 16; q++) {
+    const size_t i = base + (size_t)q * S3_THREADS + threadIdx.x;
+    if (i >= n) break;
+    ScalarReg<C> k;
+    load_scalar<C>(k, scal, i);
+    if (!scalar_in_range<C>(k)) { bad = true; continue; }
+    for_each_digit<C>(k, c, nwin, [&](int j, uint32_t b, bool) { atomicAdd(hist + ((j * ws + b) >> sh1), 1u); });
+  }
+  if (bad) atomicOr(err, 4u);
+  __syncthreads();
+  for (uint32_t i = threadIdx.x; i < NC1; i += blockDim.x)
+    if (hist[i]) atomicAdd(binCount + i, hist[i]);
+}
+
+// P1: tile = tp points (tp * nwin <= S3_TILE entries)
+template <class C>
+__global__ void __launch_bounds__(S3_THREADS) k_s3_part1(const uint32_t* __restrict__ scal, size_t n, int c, int nwin,
+                                                         uint32_t ws, uint32_t istride, int sh1, uint32_t NC1, uint32_t tp,
+                                                         uint32_t* __restrict__ binCursor,
+                                                         uint32_t* __restrict__ keys, uint32_t* __restrict__ vals) {
+  extern __shared__ uint32_t sm[];
+  uint32_t* skey = sm;                 // [S3_TILE]
+  uint32_t* sval = sm + S3_TILE;       // [S3_TILE]
+  __shared__ uint32_t loc[S3_MAXB], cur[S3_MAXB], gbase[S3_MAXB], warp_sums[32];
+  for (uint32_t i = threadIdx.x; i < NC1; i += blockDim.x) cur[i] = 0;
+  __syncthreads();
+  const size_t p0 = (size_t)blockIdx.x * tp;
+  const size_t p1 = min(p0 + tp, n);
+  for (size_t i = p0 + threadIdx.x; i < p1; i += blockDim.x) {
+    ScalarReg<C> k;
+    load_scalar<C>(k, scal, i);
+    if (!scalar_in_range<C>(k)) continue;
+    for_each_digit<C>(k, c, nwin, [&](int j, uint32_t b, bool) { atomicAdd(cur + ((j * ws + b) >> sh1), 1u); });
+  }
+  __syncthreads();
+  for (uint32_t i = threadIdx.x; i < NC1; i += blockDim.x) {
+    const uint32_t h = cur[i];
+    gbase[i] = h ? atomicAdd(binCursor + i, h) : 0u;
+    loc[i] = h;
+  }
+  __syncthreads();
+  const uint32_t E = s3_block_scan(loc, NC1, warp_sums);
+  for (uint32_t i = threadIdx.x; i < NC1; i += blockDim.x) cur[i] = loc[i];
+  __syncthreads();
+  for (size_t i = p0 + threadIdx.x; i < p1; i += blockDim.x) {
+    ScalarReg<C> k;
+    load_scalar<C>(k, scal, i);
+    if (!scalar_in_range<C>(k)) continue;
+    for_each_digit<C>(k, c, nwin, [&](int j, uint32_t b, bool neg) {
+      const uint32_t f = j * ws + b;
+      const uint32_t pos = atomicAdd(cur + (f >> sh1), 1u);
+      skey[pos] = f;
+      sval[pos] = ((uint32_t)i + (uint32_t)j * istride) | (neg ? SIGN_BIT : 0u);
+    });
+  }
+  __syncthreads();
+  for (uint32_t p = threadIdx.x; p < E; p += blockDim.x) {
+    const uint32_t f = skey[p], bin = f >> sh1;
+    const uint32_t o = gbase[bin] + (p - loc[bin]);
+    keys[o] = f;
+    vals[o] = sval[p];
+  }
+}
+
+// P2 work is cut into tiles of <= S3_TILE entries that never straddle a P1 bin, so heavy
+// bins (skewed scalars; with the f3 table the top window's small digits all land in the
+// lowest buckets) spread over many blocks.  tileStart[b] = first tile of P1 bin b.
+static __global__ void k_s3_tiles(const uint32_t* __restrict__ binOff, uint32_t NC1, uint32_t* __restrict__ tileStart) {
+  __shared__ uint32_t cnt[S3_MAXB], warp_sums[32];
+  for (uint32_t i = threadIdx.x; i < NC1; i += blockDim.x)
+    cnt[i] = (binOff[i + 1] - binOff[i] + S3_TILE - 1) / S3_TILE;
+  __syncthreads();
+  const uint32_t total = s3_block_scan(cnt, NC1, warp_sums);
+  for (uint32_t i = threadIdx.x; i < NC1; i += blockDim.x) tileStart[i] = cnt[i];
+  if (threadIdx.x == 0) tileStart[NC1] = total;
+}
+
+// tile t -> its P1 bin and entry range; false past the last tile
+__device__ __forceinline__ bool s3_tile(const uint32_t* __restrict__ tileStart, const uint32_t* __restrict__ binOff,
+                                        uint32_t NC1, uint32_t t, uint32_t& bin, uint32_t& e0, uint32_t& e1) {
+  if (t >= tileStart[NC1]) return false;
+  uint32_t lo = 0, hi = NC1;  // largest bin with tileStart[bin] <= t (tileStart non-decreasing)
+  while (hi - lo > 1) {
+    const uint32_t mid = (lo + hi) >> 1;
+    if (tileStart[mid] <= t) lo = mid; else hi = mid;
+  }
+  while (lo + 1 < NC1 && tileStart[lo + 1] <= t) lo++;  // skip empty bins sharing the start
+  bin = lo;
+  e0 = binOff[bin] + (t - tileStart[bin]) * S3_TILE;
+  e1 = min(e0 + S3_TILE, binOff[bin + 1]);
+  return true;
+}
+
+// P2 histogram: subCount[bin*NC2 + s] for s = (f >> sh2) & (NC2 - 1)
+static __global__ void __launch_bounds__(S3_THREADS) k_s3_count2(const uint32_t* __restrict__ tileStart,
+                                                                 const uint32_t* __restrict__ binOff, uint32_t NC1,
+                                                                 int sh2, uint32_t NC2, const uint32_t* __restrict__ keys,
+                                                                 uint32_t* __restrict__ subCount) {
+  __shared__ uint32_t hist[S3_MAXB];
+  uint32_t bin, e0, e1;
+  if (!s3_tile(tileStart, binOff, NC1, blockIdx.x, bin, e0, e1)) return;
+  const uint32_t mask = NC2 - 1;
+  for (uint32_t i = threadIdx.x; i < NC2; i += blockDim.x) hist[i] = 0;
+  __syncthreads();
+  for (uint32_t e = e0 + threadIdx.x; e < e1; e += blockDim.x) atomicAdd(hist + ((__ldg(keys + e) >> sh2) & mask), 1u);
+  __syncthreads();
+  for (uint32_t i = threadIdx.x; i < NC2; i += blockDim.x)
+    if (hist[i]) atomicAdd(subCount + (size_t)bin * NC2 + i, hist[i]);
+}
+
+// P2 scatter: per tile, shared-memory ranks by sub-bin, one global atomic per (tile,
+// sub-bin) on subCursor (initialised to the global sub-bin starts), staged coalesced runs.
+static __global__ void __launch_bounds__(S3_THREADS) k_s3_part2(const uint32_t* __restrict__ tileStart,
+                                                                const uint32_t* __restrict__ binOff, uint32_t NC1,
+                                                                int sh2, uint32_t NC2,
+                                                                const uint32_t* __restrict__ keys, const uint32_t* __restrict__ vals,
+                                                                uint32_t* __restrict__ subCursor,
+                                                                uint32_t* __restrict__ keys2, uint32_t* __restrict__ vals2) {
+  extern __shared__ uint32_t sm[];
+  uint32_t* skey = sm;
+  uint32_t* sval = sm + S3_TILE;
+  __shared__ uint32_t loc[S3_MAXB], cur[S3_MAXB], gbase[S3_MAXB], warp_sums[32];
+  uint32_t bin, e0, e1;
+  if (!s3_tile(tileStart, binOff, NC1, blockIdx.x, bin, e0, e1)) return;
+  const uint32_t mask = NC2 - 1;
+  for (uint32_t i = threadIdx.x; i < NC2; i += blockDim.x) cur[i] = 0;
+  __syncthreads();
+  for (uint32_t e = e0 + threadIdx.x; e < e1; e += blockDim.x) atomicAdd(cur + ((__ldg(keys + e) >> sh2) & mask), 1u);
+  __syncthreads();
+  for (uint32_t i = threadIdx.x; i < NC2; i += blockDim.x) {
+    const uint32_t h = cur[i];
+    gbase[i] = h ? atomicAdd(subCursor + (size_t)bin * NC2 + i, h) : 0u;
+    loc[i] = h;
+  }
+  __syncthreads();
+  const uint32_t E = s3_block_scan(loc, NC2, warp_sums);
+  for (uint32_t i = threadIdx.x; i < NC2; i += blockDim.x) cur[i] = loc[i];
+  __syncthreads();
+  for (uint32_t e = e0 + threadIdx.x; e < e1; e += blockDim.x) {
+    const uint32_t f = __ldg(keys + e);
+    const uint32_t pos = atomicAdd(cur + ((f >> sh2) & mask), 1u);
+    skey[pos] = f;
+    sval[pos] = __ldg(vals + e);
+  }
+  __syncthreads();
+  for (uint32_t p = threadIdx.x; p < E; p += blockDim.x) {
+    const uint32_t f = skey[p], sb = (f >> sh2) & mask;
+    const uint32_t o = gbase[sb] + (p - loc[sb]);
+    keys2[o] = f;
+    vals2[o] = sval[p];
+  }
+}
+
+// P3: block = sub-bin q covering buckets [q << b3, (q+1) << b3) of [subOff[q], end_q);
+// writes goff for its buckets (< F) and the final values in bucket order.
+static __global__ void __launch_bounds__(256) k_s3_part3(const uint32_t* __restrict__ subOff, int b3, uint32_t F,
+                                                         const uint32_t* __restrict__ keys2, const uint32_t* __restrict__ vals2,
+                                                         uint32_t* __restrict__ goff, uint32_t* __restrict__ sorted) {
+  extern __shared__ uint32_t sm[];
+  uint32_t* sval = sm;                  // [S3_CAP] staged values (bucket order)
+  uint32_t* cnt = sm + S3_CAP;          // [2^b3]
+  __shared__ uint32_t warp_sums[32];
+  const uint32_t q = blockIdx.x;
+  const uint32_t e0 = subOff[q], e1 = subOff[q + 1];  // subOff[nsub] = M
+  const uint32_t nf = 1u << b3, fmask = nf - 1, fbase = q << b3;
+  for (uint32_t i = threadIdx.x; i < nf; i += blockDim.x) cnt[i] = 0;
+  __syncthreads();
+  for (uint32_t e = e0 + threadIdx.x; e < e1; e += blockDim.x) atomicAdd(cnt + (__ldg(keys2 + e) & fmask), 1u);
+  __syncthreads();
+  s3_block_scan(cnt, nf, warp_sums);
+  for (uint32_t i = threadIdx.x; i < nf; i += blockDim.x)
+    if (fbase + i < F) goff[fbase + i] = e0 + cnt[i];
+  __syncthreads();
+  const uint32_t len = e1 - e0;
+  if (len <= (uint32_t)S3_CAP) {
+    for (uint32_t e = e0 + threadIdx.x; e < e1; e += blockDim.x) {
+      const uint32_t f = __ldg(keys2 + e);
+      sval[atomicAdd(cnt + (f & fmask), 1u)] = __ldg(vals2 + e);
+    }
+    __syncthreads();
+    for (uint32_t p = threadIdx.x; p < len; p += blockDim.x) sorted[e0 + p] = sval[p];
+  } else {  // oversized sub-bin (skewed scalars): scatter straight to global
+    for (uint32_t e = e0 + threadIdx.x; e < e1; e += blockDim.x) {
+      const uint32_t f = __ldg(keys2 + e);
+      sorted[e0 + atomicAdd(cnt + (f & fmask), 1u)] = __ldg(vals2 + e);
+    }
+  }
+}

@@ -174,11 +174,11 @@ def test_device_resident_inputs(lib):
 
 
 @pytest.mark.parametrize("name", ["bn254", "bls12_381"])
-@pytest.mark.parametrize("sort", [0, 1])
+@pytest.mark.parametrize("sort", [1, 2, 3])
 @pytest.mark.parametrize("cbits", [4, 9, 13, 16])
 def test_sort_variants(lib, name, sort, cbits):
-    """a3 two-level binned sort (default) and direct-atomic sort (ablation) both give the
-    oracle's result and the oracle's bucket sums, for bin shifts 0..> 0."""
+    """a3 variants -- direct atomics (ablation), two-level binned, three-level staged -- all
+    give the oracle's result and the oracle's bucket sums, for bin shifts 0..> 0."""
     c = CURVES[name]
     n = 700
     Ps, es, _, _ = progression(name, n, 28)
@@ -207,9 +207,36 @@ def test_large_c_binned_sort(lib):
     Ps, es, _, _ = progression(name, n, 29)
     ks = synth.words_to_ints(synth.scalars(c.r, n, 41))
     ctx = lib.Context(name, points_to_words(list(Ps), name), n=n)
-    for cbits in (20, 22):
-        ctx.set_option(lib.OPT_WINDOW_BITS, cbits)
-        assert ctx.run(synth.ints_to_words(ks, 8)) == closed(name, ks, es), cbits
+    for sort in (2, 3):
+        ctx.set_option(lib.OPT_SORT, sort)
+        for pre in (0, 1):
+            ctx.set_option(lib.OPT_PRECOMPUTE, pre)
+            for cbits in (20, 22, 24):
+                ctx.set_option(lib.OPT_WINDOW_BITS, cbits)
+                assert ctx.run(synth.ints_to_words(ks, 8)) == closed(name, ks, es), (sort, pre, cbits)
+    ctx.close()
+
+
+@pytest.mark.parametrize("kind", ["ones", "skewed", "uniform"])
+def test_staged_sort_oversized_subbins(lib, kind):
+    """Three-level staged sort with > S3_CAP entries in one sub-bin (skewed scalars take
+    the global-scatter fallback of k_s3_part3) and on uniform scalars at several c."""
+    name = "bn254"
+    c = CURVES[name]
+    n = 20000
+    Ps, es, _, _ = progression(name, n, 34)
+    ks = (synth.words_to_ints(synth.scalars(c.r, n, 62)) if kind == "uniform"
+          else synth.words_to_ints(synth.pattern_scalars(c.r, n, 7, kind)))
+    want = closed(name, ks, es)
+    ctx = lib.Context(name, points_to_words(list(Ps), name), n=n)
+    ctx.set_option(lib.OPT_SORT, 3)
+    sw = synth.ints_to_words(ks, 8)
+    for pre in (0, 1):
+        ctx.set_option(lib.OPT_PRECOMPUTE, pre)
+        for cbits in (5, 11, 16):
+            ctx.set_option(lib.OPT_WINDOW_BITS, cbits)
+            assert ctx.get_option(lib.OPT_SORT) == 3
+            assert ctx.run(sw) == want, (pre, cbits)
     ctx.close()
 
 
