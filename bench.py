@@ -106,6 +106,17 @@ class ClockSampler:
                 "power_w_max": max((float(r[2]) for r in self.rows if r[2].replace(".", "").isdigit()), default=None)}
 
 
+def ncu_traffic(curve, log2n):
+    """dram__bytes_read.sum + dram__bytes_write.sum of one k_accumulate launch, from the
+    committed ncu --set full capture of this workload (profiles/ncu_traffic.json), or None."""
+    try:
+        t = json.load(open(os.path.join(ROOT, "profiles", "ncu_traffic.json")))[f"{curve} 2^{log2n}"]
+        return {"bytes": t["read"] + t["write"], "read": t["read"], "write": t["write"],
+                "algorithmic_bytes": t.get("algorithmic"), "source": t["source"]}
+    except Exception:
+        return None
+
+
 def dist_env():
     ws = int(os.environ.get("WORLD_SIZE", "1"))
     rank = int(os.environ.get("RANK", "0"))
@@ -182,6 +193,8 @@ def main():
     ap.add_argument("--window-bits", type=int, default=0)
     ap.add_argument("--precompute", type=int, default=2, choices=[0, 1, 2],
                     help="f3 window table (PAPER.md:147): 0 off, 1 on, 2 auto (library default)")
+    ap.add_argument("--sort", type=int, default=0, choices=[0, 1, 2, 3],
+                    help="a3 variant (MSM_OPT_SORT): 0 auto, 1 direct global atomics (ablation), 2 binned, 3 staged")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--ref-sample", type=int, default=0)
     ap.add_argument("--no-e2e", action="store_true")
@@ -237,6 +250,8 @@ def main():
         ctx.set_option(msm.OPT_PRECOMPUTE, args.precompute)
     if args.window_bits:
         ctx.set_option(msm.OPT_WINDOW_BITS, args.window_bits)
+    if args.sort:
+        ctx.set_option(msm.OPT_SORT, args.sort)
     setup_s = time.time() - t0
     stream = torch.cuda.ExternalStream(ctx.stream(0), device=dev)
     pw = msm.partial_words(curve)
@@ -342,7 +357,7 @@ def main():
         "config": {"workload": f"{curve} G1 MSM n=2^{args.log2n} (BASELINE.json config C4)" if (curve, args.log2n) == ("bls12_381", 26)
                    else f"{curve} G1 MSM n=2^{args.log2n}",
                    "curve": curve, "n": n, "window_bits": st["window_bits"], "nwin": st["nwin"],
-                   "precompute": bool(st["precompute"]),
+                   "precompute": bool(st["precompute"]), "sort_variant": ctx.get_option(msm.OPT_SORT),
                    "bucket_sets": 1 if st["precompute"] else st["nwin"],
                    "parallelism": f"point-sharded x{ws}" + (" + NCCL all-gather of partials" if ws > 1 else ""),
                    "scalars": "device-resident (HBM) for value; pinned host for e2e",
@@ -351,7 +366,7 @@ def main():
         "stages_ms": {k: round(v, 3) for k, v in st.items() if k.endswith("_ms") and k != "table_ms"},
         "latency_ms": {"mean": ms, "min": min(times), "max": max(times)},
         "roofline": {"kernel": "k_accumulate", "bound": "alu", "achieved": achieved / 1e12, "peak": peak_slots / 1e12,
-                     "unit": "T IMAD-pipe slots/s", "frac": achieved / peak_slots, "traffic": None,
+                     "unit": "T IMAD-pipe slots/s", "frac": achieved / peak_slots, "traffic": ncu_traffic(curve, args.log2n),
                      "work": f"{pacc} PACC x (8 mul x {imad_slots_per_mult(L)} + 2 sqr x {imad_slots_per_sqr(L)}) IMAD slots",
                      "peak_basis": f"148 SM x 64 IMAD slots/clk x {sm_max} MHz (clocks.max.sm); IMAD.WIDE = 2 slots (measured)",
                      "field_mults_per_s": pacc * 10 / (acc_avg_ms / 1e3)},

@@ -177,6 +177,29 @@ DEVI void fmul2_cols(uint32_t* r1, const uint32_t* a1, const uint32_t* b1, const
     fmul2_cols<C, SQR, K + 1>(r1, a1, b1, a21, m1, cA1, cM1, r2, a2, b2, a22, m2, cA2, cM2);
 }
 
+// Three independent products column-interleaved (six accumulation chains in split
+// columns): the PACC groups {PPP, Q, ZZ'} and {ZZZ', T, E} each need only values of the
+// previous group, so a warp can keep three products in flight (ILP at 2 warps/scheduler).
+template <class C, int K>
+DEVI void fmul3_cols(uint32_t* r1, const uint32_t* a1, const uint32_t* b1, uint32_t* m1, u64 cA1, u64 cM1,
+                     uint32_t* r2, const uint32_t* a2, const uint32_t* b2, uint32_t* m2, u64 cA2, u64 cM2,
+                     uint32_t* r3, const uint32_t* a3, const uint32_t* b3, uint32_t* m3, u64 cA3, u64 cM3) {
+  fmul_step<C, false, false, K>(r1, a1, b1, a1, m1, cA1, cM1);
+  fmul_step<C, false, false, K>(r2, a2, b2, a2, m2, cA2, cM2);
+  fmul_step<C, false, false, K>(r3, a3, b3, a3, m3, cA3, cM3);
+  if constexpr (K + 1 < 2 * C::L - 1)
+    fmul3_cols<C, K + 1>(r1, a1, b1, m1, cA1, cM1, r2, a2, b2, m2, cA2, cM2, r3, a3, b3, m3, cA3, cM3);
+}
+
+// r1 = a1*b1, r2 = a2*b2, r3 = a3*b3 (same contract as fmul; each r may alias its OWN inputs only)
+template <class C>
+DEVI void fmul3(uint32_t* r1, const uint32_t* a1, const uint32_t* b1, uint32_t* r2, const uint32_t* a2,
+                const uint32_t* b2, uint32_t* r3, const uint32_t* a3, const uint32_t* b3) {
+  constexpr int L = C::L;
+  uint32_t m1[L], m2[L], m3[L];
+  fmul3_cols<C, 0>(r1, a1, b1, m1, 0ull, 0ull, r2, a2, b2, m2, 0ull, 0ull, r3, a3, b3, m3, 0ull, 0ull);
+}
+
 template <class C, bool SQR, bool LAT = false>
 DEVI void fmul_impl(uint32_t* r, const uint32_t* a, const uint32_t* b) {
   constexpr int L = C::L;

@@ -572,6 +572,15 @@ DEVI bool point_for_entry(uint32_t* x, uint32_t* y, const uint32_t* __restrict__
 #ifndef MSM_ACC_PREFETCH
 #define MSM_ACC_PREFETCH 1
 #endif
+#ifndef MSM_ACC_PADD
+#define MSM_ACC_PADD 0  // f4 ablation: PADD (Alg. 1) with Z = 1 operand instead of PACC (Alg. 4)
+#endif
+#ifndef MSM_ACC_SMEM
+#define MSM_ACC_SMEM 0  // A/B: k_accumulate_smem (operands in shared-memory slots, one fmul2 body)
+#endif
+#ifndef MSM_ACC_TRIPLE
+#define MSM_ACC_TRIPLE 0  // k_accumulate: PACC in groups 2,2,3,3 (xyzz_acc_hot3) instead of 5 pairs
+#endif
 #ifndef MSM_ACC_DUAL
 #define MSM_ACC_DUAL 1  // k_accumulate: column-interleaved multiplication pairs (xyzz_acc_hot)
 #endif
@@ -648,8 +657,14 @@ __global__ void __launch_bounds__(128, MSM_ACC_MINB) k_accumulate(const uint32_t
       do { f++; end = __ldg(goff + f + 1); } while (end <= e);
       acc_start<C>(acc, x, y, ok);
     } else if (ok) {
-#if MSM_ACC_DUAL
-      if (xyzz_acc_hot<C>(acc, x, y)) {  // rare: the point equals the accumulator
+#if MSM_ACC_PADD
+      {  // f4 ablation (Fig. 12): general PADD (Alg. 1, 14 mults) instead of PACC
+        Xyzz<C> Pt;
+        xyzz_from_affine<C>(Pt, x, y);
+        xyzz_add<C>(acc, acc, Pt);
+      }
+#elif MSM_ACC_DUAL
+      if (MSM_ACC_TRIPLE ? xyzz_acc_hot3<C>(acc, x, y) : xyzz_acc_hot<C>(acc, x, y)) {  // rare: the point equals the accumulator
         Xyzz<C> T = acc;
         xyzz_dbl<C>(acc, T);
       }
@@ -660,6 +675,234 @@ __global__ void __launch_bounds__(128, MSM_ACC_MINB) k_accumulate(const uint32_t
   }
   if (head) { store_xyzz<C>(carry_pts + (size_t)t * XW, acc); my_carry = (int32_t)f; }
   else store_xyzz<C>(buckets + (size_t)f * XW, acc);
+  carry_f[t] = my_carry;
+}
+
+// ---------------------------------------------------------------------------------------
+// a4 variant (MSM_ACC_SMEM, A/B): the PAPER.md:267 idea — big integers cached in shared
+// memory instead of registers — taken to its end.  The accumulator and every PACC
+// temporary live in per-thread shared-memory slots; the ten multiplications are five
+// steps of ONE column-interleaved fmul2 body (squarings as multiplications) whose operands
+// are loaded from slots chosen per step, so the hot loop is a few KB of code instead of
+// ~100 KB (ncu: no_instruction is the second stall of k_accumulate) and needs far fewer
+// registers.  Slot layout: word (slot*L + i) of thread t at smem[(slot*L + i)*ACC_NT + t].
+constexpr int ACC_NT = 128;
+constexpr int ACC_SLOTS = 10;  // X Y ZZ ZZZ P R PP V PPP Q
+enum { SX = 0, SY, SZZ, SZZZ, SP, SR, SPP, SV, SPPP, SQ };
+
+// operand slots (a1, b1, a2, b2) of the step program, 4 bits each: steps 0-4 are PACC
+// (Alg. 4), steps 5-9 the doubling dbl-2008-s-1 (a = 0 curves) for the rare acc == P case
+static __constant__ uint32_t ACC_OPS[10] = {
+    (SPPP) | (SZZ << 4) | (SQ << 8) | (SZZZ << 12),
+    (SP) | (SP << 4) | (SR << 8) | (SR << 12),
+    (SPP) | (SP << 4) | (SX << 8) | (SPP << 12),
+    (SZZ) | (SPP << 4) | (SY << 8) | (SPPP << 12),
+    (SZZZ) | (SPPP << 4) | (SR << 8) | (SQ << 12),
+    (SP) | (SP << 4) | (SX << 8) | (SX << 12),
+    (SP) | (SR << 4) | (SX << 8) | (SR << 12),
+    (SR) | (SZZ << 4) | (SV << 8) | (SZZZ << 12),
+    (SV) | (SY << 4) | (SQ << 8) | (SQ << 12),
+    (SQ) | (SPP << 4) | (SQ << 8) | (SQ << 12)};
+
+template <class C>
+DEVI void sload(uint32_t* v, const uint32_t* sb, int slot) {
+#pragma unroll
+  for (int i = 0; i < C::L; i++) v[i] = sb[(slot * C::L + i) * ACC_NT];
+}
+template <class C>
+DEVI void sstore(uint32_t* sb, int slot, const uint32_t* v) {
+#pragma unroll
+  for (int i = 0; i < C::L; i++) sb[(slot * C::L + i) * ACC_NT] = v[i];
+}
+template <class C>
+DEVI void sload_xyzz(Xyzz<C>& A, const uint32_t* sb) {
+  sload<C>(A.X, sb, SX); sload<C>(A.Y, sb, SY); sload<C>(A.ZZ, sb, SZZ); sload<C>(A.ZZZ, sb, SZZZ);
+}
+template <class C>
+DEVI void sstore_xyzz(uint32_t* sb, const Xyzz<C>& A) {
+  sstore<C>(sb, SX, A.X); sstore<C>(sb, SY, A.Y); sstore<C>(sb, SZZ, A.ZZ); sstore<C>(sb, SZZZ, A.ZZZ);
+}
+template <class C>
+DEVI bool s_is_zero(const uint32_t* sb, int slot) {
+  uint32_t v[C::L];
+  sload<C>(v, sb, slot);
+  return fis_zero<C, 2>(v);
+}
+
+// acc(slots X..ZZZ) += (x, y) held in slots PPP, Q: Alg. 4 with the bounds of
+// xyzz_acc_hot, as a program of multiplication pairs through ONE fmul2 body.
+//   step 0  U2 = x ZZ,  S2 = y ZZZ       P = U2 - X, R = S2 - Y (zero tests)
+//   step 1  PP = P P,   V = R R
+//   step 2  PPP = PP P, Q = X PP          X' = V - PPP - 2Q, D = Q - X'
+//   step 3  ZZ' = ZZ PP, T = Y PPP
+//   step 4  ZZZ' = ZZZ PPP, E = R D       Y' = E - T
+// acc == (x, y) (P = R = 0) continues with the doubling of acc (xyzz_dbl's formula/bounds):
+//   pre     U = 2Y                        (< 8p)
+//   step 5  V = U U,    X^2 = X X
+//   step 6  W = U V,    S = X V           M = 3 X^2
+//   step 7  ZZ' = V ZZ, ZZZ' = W ZZZ
+//   step 8  WY = W Y,   M^2               X' = M^2 - 2S, D = S - X'
+//   step 9  E = M D     (pair slot idle)  Y' = E - WY
+template <class C>
+DEVI void s_pacc(uint32_t* sb) {
+  constexpr int L = C::L;
+  static_assert(C::A_ZERO, "smem step program: a = 0 curves");
+  // the step bounds are opaque to the optimiser, so the loop stays a loop (one fmul2 body)
+  int step, stop;
+  asm volatile("mov.u32 %0, 0;" : "=r"(step));
+  asm volatile("mov.u32 %0, 5;" : "=r"(stop));
+#pragma unroll 1
+  for (; step < stop; step++) {
+    const uint32_t ops = ACC_OPS[step];
+    uint32_t a1[L], b1[L], a2[L], b2[L], r1[L], r2[L];
+    sload<C>(a1, sb, ops & 15);
+    sload<C>(b1, sb, (ops >> 4) & 15);
+    sload<C>(a2, sb, (ops >> 8) & 15);
+    sload<C>(b2, sb, (ops >> 12) & 15);
+    fmul2<C>(r1, a1, b1, r2, a2, b2);
+    switch (step) {
+      case 0:
+        sload<C>(a1, sb, SX);
+        sload<C>(a2, sb, SY);
+        fsub<C, 8>(r1, r1, a1);  // P = U2 - X    < 10p
+        fsub<C, 4>(r2, r2, a2);  // R = S2 - Y    < 6p
+        if (fis_zero<C, 10>(r1)) {
+          if (fis_zero<C, 6>(r2)) {  // acc == (x, y): double acc instead
+            fadd<C>(b1, a2, a2);     // U = 2Y < 8p
+            sstore<C>(sb, SP, b1);
+            step = 4;
+            stop = 10;
+          } else {                   // acc == -(x, y): O
+            fzero<C>(a1);
+#pragma unroll
+            for (int q = 0; q < 4; q++) sstore<C>(sb, q, a1);
+            stop = 0;
+          }
+          break;
+        }
+        sstore<C>(sb, SP, r1);
+        sstore<C>(sb, SR, r2);
+        break;
+      case 1:
+        sstore<C>(sb, SPP, r1);  // PP < 2p
+        sstore<C>(sb, SV, r2);   // V  < 2p
+        break;
+      case 2:
+        sload<C>(a1, sb, SV);
+        fadd<C>(b1, r1, r2);
+        fadd<C>(b1, b1, r2);     // PPP + 2Q      < 6p
+        fsub<C, 6>(b2, a1, b1);  // X' = V - PPP - 2Q < 8p
+        fsub<C, 8>(a2, r2, b2);  // D = Q - X'    < 10p
+        sstore<C>(sb, SPPP, r1);
+        sstore<C>(sb, SX, b2);
+        sstore<C>(sb, SQ, a2);
+        break;
+      case 3:
+        sstore<C>(sb, SZZ, r1);  // ZZ' < 2p
+        sstore<C>(sb, SV, r2);   // T   < 2p
+        break;
+      case 4:
+        sload<C>(a1, sb, SV);
+        fsub<C, 2>(b1, r2, a1);  // Y' = E - T    < 4p
+        sstore<C>(sb, SZZZ, r1);
+        sstore<C>(sb, SY, b1);
+        break;
+      case 5:
+        sstore<C>(sb, SR, r1);   // V = U^2 < 2p
+        sstore<C>(sb, SPP, r2);  // X^2 < 2p
+        break;
+      case 6:
+        sstore<C>(sb, SV, r1);    // W = U V < 2p
+        sstore<C>(sb, SPPP, r2);  // S = X V < 2p
+        sload<C>(a1, sb, SPP);
+        fadd<C>(b1, a1, a1);
+        fadd<C>(b1, b1, a1);      // M = 3 X^2 < 6p
+        sstore<C>(sb, SQ, b1);
+        break;
+      case 7:
+        sstore<C>(sb, SZZ, r1);   // ZZ' = V ZZ < 2p
+        sstore<C>(sb, SZZZ, r2);  // ZZZ' = W ZZZ < 2p
+        break;
+      case 8:
+        sstore<C>(sb, SR, r1);    // WY < 2p
+        sload<C>(a1, sb, SPPP);   // S
+        fadd<C>(b1, a1, a1);      // 2S < 4p
+        fsub<C, 4>(b2, r2, b1);   // X' = M^2 - 2S < 6p
+        fsub<C, 6>(a2, a1, b2);   // D = S - X' < 8p
+        sstore<C>(sb, SX, b2);
+        sstore<C>(sb, SPP, a2);
+        break;
+      default:
+        sload<C>(a1, sb, SR);
+        fsub<C, 2>(b1, r1, a1);   // Y' = M D - WY < 4p
+        sstore<C>(sb, SY, b1);
+        break;
+    }
+  }
+}
+
+template <class C>
+DEVI void s_start(uint32_t* sb, const uint32_t* x, const uint32_t* y, bool ok) {
+  Xyzz<C> A;
+  if (ok) xyzz_from_affine<C>(A, x, y);
+  else xyzz_set_zero<C>(A);
+  sstore_xyzz<C>(sb, A);
+}
+
+template <class C>
+__global__ void __launch_bounds__(ACC_NT, MSM_ACC_MINB) k_accumulate_smem(const uint32_t* __restrict__ pts, const uint32_t* __restrict__ sorted,
+                                                    const uint32_t* __restrict__ goff, uint32_t F,
+                                                    uint32_t* __restrict__ buckets, uint32_t* __restrict__ carry_pts,
+                                                    int32_t* __restrict__ carry_f, uint32_t nthreads,
+                                                    uint32_t* __restrict__ nlong) {
+  constexpr int XW = Layout<C>::XW;
+  extern __shared__ uint32_t acc_smem[];
+  uint32_t* sb = acc_smem + threadIdx.x;
+  const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+  if (t == 0) *nlong = 0;
+  if (t >= nthreads) return;
+  const uint32_t M = __ldg(goff + F);
+  const uint32_t slice = M ? (M + nthreads - 1) / nthreads : 1u;
+  const uint64_t e0l = (uint64_t)t * slice;
+  if (e0l >= M) { carry_f[t] = -1; return; }
+  const uint32_t e0 = (uint32_t)e0l;
+  const uint32_t e1 = (uint32_t)(e0l + slice < (uint64_t)M ? e0l + slice : (uint64_t)M);
+  uint32_t f = find_bucket(goff, F, e0);
+  uint32_t end = __ldg(goff + f + 1);
+  bool head = __ldg(goff + f) < e0;
+  uint32_t x[C::L], y[C::L];
+  bool ok = point_for_entry<C>(x, y, pts, __ldg(sorted + e0));
+  s_start<C>(sb, x, y, ok);
+  int32_t my_carry = -1;
+  uint32_t ent1 = e0 + 1 < e1 ? __ldg(sorted + e0 + 1) : 0u;
+  uint32_t ent2 = e0 + 2 < e1 ? __ldg(sorted + e0 + 2) : 0u;
+  if (e0 + 1 < e1) prefetch_point<C>(pts, ent1);
+  Xyzz<C> A;
+  for (uint32_t e = e0 + 1; e < e1; e++) {
+    const uint32_t ent = ent1;
+    ent1 = ent2;
+    if (e + 1 < e1) prefetch_point<C>(pts, ent1);
+    if (e + 2 < e1) ent2 = __ldg(sorted + e + 2);
+    ok = point_for_entry<C>(x, y, pts, ent);
+    if (e == end) {
+      sload_xyzz<C>(A, sb);
+      if (head) { store_xyzz<C>(carry_pts + (size_t)t * XW, A); my_carry = (int32_t)f; head = false; }
+      else store_xyzz<C>(buckets + (size_t)f * XW, A);
+      do { f++; end = __ldg(goff + f + 1); } while (end <= e);
+      s_start<C>(sb, x, y, ok);
+    } else if (ok) {
+      if (s_is_zero<C>(sb, SZZ)) {
+        s_start<C>(sb, x, y, true);
+      } else {
+        sstore<C>(sb, SPPP, x);
+        sstore<C>(sb, SQ, y);
+        s_pacc<C>(sb);
+      }
+    }
+  }
+  sload_xyzz<C>(A, sb);
+  if (head) { store_xyzz<C>(carry_pts + (size_t)t * XW, A); my_carry = (int32_t)f; }
+  else store_xyzz<C>(buckets + (size_t)f * XW, A);
   carry_f[t] = my_carry;
 }
 

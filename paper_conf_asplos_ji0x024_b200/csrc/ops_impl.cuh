@@ -101,7 +101,13 @@ struct Ops final : CurveOps {
     const int sms = prop.multiProcessorCount;
     s.sms = sms;
     int bps = 0;
+#if MSM_ACC_SMEM
+    constexpr int acc_smem = ACC_SLOTS * C::L * ACC_NT * 4;
+    CK(cudaFuncSetAttribute(k_accumulate_smem<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, acc_smem));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_accumulate_smem<C>, 128, acc_smem));
+#else
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_accumulate<C>, 128, 0));
+#endif
     if (bps < 1) bps = 1;
     const size_t resident = (size_t)sms * bps * 128;
     const size_t Mmax = s.n * (size_t)s.nwin;
@@ -259,7 +265,11 @@ struct Ops final : CurveOps {
     CK(cudaGetLastError());
     if (timed) CK(cudaEventRecord(s.ev[EV_SORT], st));
     // a4: accumulate + fixup
+#if MSM_ACC_SMEM
+    k_accumulate_smem<C><<<(unsigned)cdiv(s.acc_threads, 128), 128, ACC_SLOTS * C::L * ACC_NT * 4, st>>>(pts, s.sorted, s.goff, (uint32_t)s.F,
+#else
     k_accumulate<C><<<(unsigned)cdiv(s.acc_threads, 128), 128, 0, st>>>(pts, s.sorted, s.goff, (uint32_t)s.F,
+#endif
                                                                         s.buckets, s.carry_pts, s.carry_f, s.acc_threads,
                                                                         s.nlong);
     launches++;

@@ -22,7 +22,7 @@ if a.names:
 for lib in libs:
     env = dict(os.environ, MSM_LIB=lib)
     cmd = [sys.executable, os.path.join(ROOT, "bench.py"), "--log2n", str(a.log2n), "--curve", a.curve, "--steps",
-           str(a.steps), "--no-e2e", "--no-cpu-baseline"]
+           str(a.steps), "--no-e2e", "--no-cpu-baseline", "--check"]
     if a.window_bits:
         cmd += ["--window-bits", str(a.window_bits)]
     r = subprocess.run(cmd, env=env, capture_output=True, text=True)
@@ -35,4 +35,5 @@ for lib in libs:
     st = d["stages_ms"]
     print(json.dumps({"variant": name, "ms": round(d["ms_per_step"], 2), "acc_ms": st["accumulate_ms"],
                       "sort_ms": st["sort_ms"], "reduce_ms": st["reduce_ms"], "combine_ms": st["combine_ms"],
-                      "frac": round(d["roofline"]["frac"], 4), "c": d["config"]["window_bits"]}), flush=True)
+                      "frac": round(d["roofline"]["frac"], 4), "c": d["config"]["window_bits"],
+                      "check": d.get("check")}), flush=True)

@@ -2,6 +2,7 @@
 # Build BLS12-381-only variant libraries for A/B timing (other curves reuse build/ objects).
 set -e
 cd "$(dirname "$0")/.."
+mkdir -p variants
 build_variant() {  # name, defines...
   name=$1; shift
   args=()

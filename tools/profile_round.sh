@@ -11,4 +11,5 @@ for k in ${KERNELS:-k_accumulate k_bucket_segments k_s3_scatter}; do
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:$k -s 1 -c 1 -o $o/$k -f $B > $o/$k.log 2>&1
   ncu -i $o/$k.ncu-rep --page raw --csv > $o/${k}_raw.csv 2>/dev/null
   ncu -i $o/$k.ncu-rep --page details --csv > $o/${k}_details.csv 2>/dev/null
+  rm -f $o/$k.ncu-rep  # reports are tens of MB; gpurun copies back <= 64 MiB
 done
