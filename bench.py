@@ -195,6 +195,9 @@ def main():
                     help="f3 window table (PAPER.md:147): 0 off, 1 on, 2 auto (library default)")
     ap.add_argument("--sort", type=int, default=0, choices=[0, 1, 2, 3],
                     help="a3 variant (MSM_OPT_SORT): 0 auto, 1 direct global atomics (ablation), 2 binned, 3 staged")
+    ap.add_argument("--split", default="auto", choices=["auto", "points", "buckets"],
+                    help="N > 1 decomposition: point shards, or the paper's bucket split (PAPER.md:223); "
+                         "auto = buckets for N > 1")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--ref-sample", type=int, default=0)
     ap.add_argument("--no-e2e", action="store_true")
@@ -231,7 +234,11 @@ def main():
     L32, S, lam, L, W = CURVE_INFO[curve]
     r = synth.CURVE_ORDERS[curve]
     n = 1 << args.log2n
-    off, n_g = shard_bounds(n, ws, rank)
+    # multi-GPU decomposition: "points" = contiguous point shards (north_star), "buckets" =
+    # the paper's bucket split (f1): every rank holds all n points and scalars
+    # and sums the buckets |d| = ws*q + rank of every bucket set
+    split = args.split if args.split != "auto" else ("buckets" if ws > 1 else "points")
+    off, n_g = shard_bounds(n, ws, rank) if split == "points" else (0, n)
     seed = 20240427 + 3
     e0, delta = synth.point_seeds(r, seed)
 
@@ -252,6 +259,9 @@ def main():
         ctx.set_option(msm.OPT_WINDOW_BITS, args.window_bits)
     if args.sort:
         ctx.set_option(msm.OPT_SORT, args.sort)
+    if split == "buckets" and ws > 1:
+        ctx.set_option(msm.OPT_SPLIT_PARTS, ws)
+        ctx.set_option(msm.OPT_SPLIT_INDEX, rank)
     setup_s = time.time() - t0
     stream = torch.cuda.ExternalStream(ctx.stream(0), device=dev)
     pw = msm.partial_words(curve)
@@ -312,7 +322,7 @@ def main():
             torch.distributed.all_reduce(e_t, op=torch.distributed.ReduceOp.MAX)
         e2e_ms = float(e_t.item())
         e2e = {"value": n / (e2e_ms / 1e3), "unit": "points/s", "ms_per_step": e2e_ms,
-               "h2d_bytes_per_step": n * S * 4, "d2h_bytes_per_step": 2 * L32 * 4,
+               "h2d_bytes_per_step": (n if split == "points" else n * ws) * S * 4, "d2h_bytes_per_step": 2 * L32 * 4,
                "timing": "host wall clock around msm_run with pinned host scalars (max over ranks)"}
 
     check = None
@@ -336,6 +346,13 @@ def main():
     sm_max = pk.get("sm_max_mhz", 1965.0)
     peak_slots = 148 * 64 * sm_max * 1e6
     achieved = slots / (acc_avg_ms / 1e3)
+    # a3 (digits + counting sort) against HBM: algorithmic bytes = scalars read once
+    # (n*S*4) + sorted entries written once (M*4); sort_ms is the stage's CUDA-event time on
+    # the library stream
+    sort_ms = sum(x["sort_ms"] for x in stage) / len(stage)
+    sort_bytes = n_g * S * 4 + int(st["entries"]) * 4
+    hbm_peak = pk.get("hbm_gbs", 6550.0)
+    sort_gbs = sort_bytes / (sort_ms / 1e3) / 1e9 if sort_ms > 0 else None
     clocks = sampler.summary()
     cpu = None
     if not args.no_cpu_baseline and ws == 1:
@@ -359,10 +376,16 @@ def main():
                    "curve": curve, "n": n, "window_bits": st["window_bits"], "nwin": st["nwin"],
                    "precompute": bool(st["precompute"]), "sort_variant": ctx.get_option(msm.OPT_SORT),
                    "bucket_sets": 1 if st["precompute"] else st["nwin"],
-                   "parallelism": f"point-sharded x{ws}" + (" + NCCL all-gather of partials" if ws > 1 else ""),
+                   "parallelism": (f"point-sharded x{ws}" if split == "points" else f"bucket-split x{ws} (PAPER.md:223)")
+                                  + (" + NCCL all-gather of partials" if ws > 1 else ""),
                    "scalars": "device-resident (HBM) for value; pinned host for e2e",
                    "l2": "inputs >> L2 (points %.1f GB + scalars %.1f GB per step); no flush needed" % (
                        n * (2 * L + 2) * 4 / 1e9, n * S * 4 / 1e9)},
+        "roofline_sort": {"stage": "a3 digits + counting sort (all kernels between EV_H2D and EV_SORT)", "bound": "hbm",
+                          "achieved": sort_gbs, "peak": hbm_peak, "unit": "GB/s",
+                          "frac": (sort_gbs / hbm_peak) if sort_gbs else None, "traffic": None,
+                          "work": f"{n_g} x {S * 4} B scalars + {int(st['entries'])} x 4 B sorted entries per step",
+                          "peak_basis": "MEASURED_PEAKS.json hbm_gbs (copy bandwidth)"},
         "stages_ms": {k: round(v, 3) for k, v in st.items() if k.endswith("_ms") and k != "table_ms"},
         "latency_ms": {"mean": ms, "min": min(times), "max": max(times)},
         "roofline": {"kernel": "k_accumulate", "bound": "alu", "achieved": achieved / 1e12, "peak": peak_slots / 1e12,

@@ -68,6 +68,15 @@ enum {
                                  With it all windows share one bucket set; building the table
                                  costs ~c*nwin doublings per point at create / option change;
                                  get returns the mode in use (0/1).                          */
+  MSM_OPT_SPLIT_PARTS = 6,    /* f1 bucket split (§3.2.2: "splits the buckets
+                                 into GPUs-per-window parts"): G in [1, 256], default 1.  With
+                                 G > 1 this context sums only the buckets |d| = G*q + g
+                                 (g = MSM_OPT_SPLIT_INDEX) of every bucket set, over ALL n points
+                                 and scalars; msm_run_partial then returns that part's share and
+                                 msm_finalize over the G parts' partials gives the MSM.  The
+                                 interleaved (b mod G) assignment balances the parts even though
+                                 the top window's digits sit in low buckets.                  */
+  MSM_OPT_SPLIT_INDEX = 7,    /* f1: this context's part g in [0, G), default 0               */
   MSM_OPT_NWIN = 101,         /* (get only) number of windows floor(lambda/c) + 1           */
   MSM_OPT_NSETS = 103,        /* (get only) bucket sets: nwin, or 1 with the f3 table        */
   MSM_OPT_NONEMPTY = 102      /* (get only) non-empty buckets of the last run on device 0   */

@@ -125,3 +125,30 @@ def bucket_sums_precomputed(ks, Ps, c, curve):
 def msm_precomputed(ks, Ps, c, curve):
     """Q = sum_b b * B^pre_b (a single bucket-reduce)."""
     return window_sums([bucket_sums_precomputed(ks, Ps, c, curve)], curve)[0]
+
+
+def bucket_split_partial(ks, Ps, c, curve, G, g, pre=False):
+    """Part g of G of the bucket split (§3.2.2: DistMSM "splits the buckets
+    into GPUs-per-window parts"; each GPU reduces only its buckets and the CPU adds the
+    N_gpu results).  Part g owns the buckets b = |d| with b mod G = g
+    (reading R18: interleaved, so the top window's small digits spread over all
+    parts).  Written from the definitions, not the running sum:
+        without the table:  sum_j 2^(j c) * sum_{b mod G = g} b * B_{j,b}
+        with it (pre):      sum_{b mod G = g} b * B^pre_b
+    The G parts sum to Q."""
+    if pre:
+        B = bucket_sums_precomputed(ks, Ps, c, curve)
+        Q = None
+        for b in range(1, len(B)):
+            if b % G == g:
+                Q = ec.add(Q, ec.mul(b, B[b], curve), curve)
+        return Q
+    Bw = bucket_sums(ks, Ps, c, curve)
+    Q = None
+    for j, Bj in enumerate(Bw):
+        Wj = None
+        for b in range(1, len(Bj)):
+            if b % G == g:
+                Wj = ec.add(Wj, ec.mul(b, Bj[b], curve), curve)
+        Q = ec.add(Q, ec.mul(1 << (j * c), Wj, curve), curve)
+    return Q

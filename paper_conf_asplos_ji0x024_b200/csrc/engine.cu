@@ -478,6 +478,15 @@ int msm_set_option(msm_context* ctx, int key, long value) {
       if (value < 0 || value > 2) return MSM_ERR_ARG;
       ctx->opt.pre = (int)value;
       break;
+    case MSM_OPT_SPLIT_PARTS:
+      if (value < 1 || value > 256) return MSM_ERR_ARG;
+      ctx->opt.split_G = (int)value;
+      if (ctx->opt.split_g >= ctx->opt.split_G) ctx->opt.split_g = 0;
+      break;
+    case MSM_OPT_SPLIT_INDEX:
+      if (value < 0 || value >= ctx->opt.split_G) return MSM_ERR_ARG;
+      ctx->opt.split_g = (int)value;
+      break;
     default:
       return MSM_ERR_ARG;
   }
@@ -494,6 +503,8 @@ long msm_get_option(msm_context* ctx, int key) {
     case MSM_OPT_NWIN: return ctx->shards[0].nwin;
     case MSM_OPT_PRECOMPUTE: return ctx->shards[0].pre;
     case MSM_OPT_NSETS: return ctx->shards[0].nset;
+    case MSM_OPT_SPLIT_PARTS: return ctx->opt.split_G;
+    case MSM_OPT_SPLIT_INDEX: return ctx->opt.split_g;
     case MSM_OPT_NONEMPTY: {
       long v = MSM_ERR_CUDA;
       guarded([&]() -> int { CK(cudaSetDevice(ctx->shards[0].dev)); v = ctx->ops->count_nonempty(ctx->shards[0]); return MSM_OK; });

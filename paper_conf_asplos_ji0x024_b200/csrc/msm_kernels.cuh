@@ -261,8 +261,13 @@ DEVI uint32_t scalar_bits(const ScalarReg<C>& k, int bit, int c) {
 }
 
 // Walks the windows of one scalar, calling f(j, bucket, negative) for non-zero digits.
+// cp = c | (G - 1) << 8 | g << 16 packs the f1 bucket split ("splits the
+// buckets into GPUs-per-window parts"): with G > 1 only digits |d| = G*q + g are emitted,
+// as local bucket q (weight G*q + g in the bucket reduce).  G = 1: every digit, bucket |d|.
 template <class C, class F>
-DEVI void for_each_digit(const ScalarReg<C>& k, int c, int nwin, F&& f) {
+DEVI void for_each_digit(const ScalarReg<C>& k, int cp, int nwin, F&& f) {
+  const int c = cp & 0xff;
+  const uint32_t G = ((uint32_t)(cp >> 8) & 0xffu) + 1u, g = (uint32_t)(cp >> 16) & 0xffu;
   const uint32_t half = 1u << (c - 1);
   uint32_t carry = 0;
   for (int j = 0; j < nwin; j++) {
@@ -275,7 +280,12 @@ DEVI void for_each_digit(const ScalarReg<C>& k, int c, int nwin, F&& f) {
     } else {
       carry = 0;
     }
-    if (d) f(j, d, neg);
+    if (G == 1) {
+      if (d) f(j, d, neg);
+    } else if (d >= g && d != 0) {
+      const uint32_t q = (d - g) / G;
+      if (q * G + g == d) f(j, q, neg);
+    }
   }
 }
 
@@ -1034,31 +1044,41 @@ DEVI void xyzz_mul_small(Xyzz<C>& R, const Xyzz<C>& A, uint32_t k, int bits) {
   }
 }
 
+// Segment t of set j covers local buckets [lo, lo + seg), lo = t*seg, of the NB local
+// buckets 0..NB-1 (bucket q has weight alpha*q + beta: alpha = 1, beta = 0 without the f1
+// split, alpha = G, beta = g with it).  Descending running sums give
+//   run = sum_q B_q,   tri = sum_q (q - lo) B_q          (2 PADD per bucket)
+// and the segment's share of W_j = sum_q (alpha q + beta) B_q is
+//   alpha*tri + (alpha*lo + beta)*run.
 template <class C>
 __global__ void __launch_bounds__(128, MSM_SEG_MINB) k_bucket_segments(const uint32_t* __restrict__ buckets, const uint32_t* __restrict__ goff,
                                                          int nwin, uint32_t NB, uint32_t seg, uint32_t nseg,
+                                                         uint32_t alpha, uint32_t beta,
                                                          uint32_t* __restrict__ out) {
   constexpr int XW = Layout<C>::XW;
   const uint32_t gid = blockIdx.x * blockDim.x + threadIdx.x;
   if (gid >= (uint32_t)nwin * nseg) return;
   const uint32_t j = gid / nseg, t = gid % nseg;
-  const uint32_t nb = NB - 1;  // buckets 1..nb
-  const uint32_t lo = 1 + t * seg;
+  const uint32_t lo = t * seg;
   Xyzz<C> run, tri, B;
   xyzz_set_zero<C>(run);
   xyzz_set_zero<C>(tri);
-  // uniform trip count `seg`; buckets past nb and empty buckets contribute O
+  // uniform trip count `seg`; buckets past NB - 1 and empty buckets contribute O
   for (uint32_t q = seg; q-- > 0;) {
     const uint32_t b = lo + q;
     const size_t f = (size_t)j * NB + b;
-    const bool ne = b <= nb && __ldg(goff + f + 1) != __ldg(goff + f);
+    const bool ne = b < NB && __ldg(goff + f + 1) != __ldg(goff + f);
     if (ne) load_xyzz<C>(B, buckets + f * XW);
     else xyzz_set_zero<C>(B);
     xyzz_add_hot<C>(run, run, B);
-    xyzz_add_hot<C>(tri, tri, run);
+    if (q > 0) xyzz_add_hot<C>(tri, tri, run);  // warp-uniform: q is the same in every lane
   }
-  int bits = 32 - __clz(nb);
-  xyzz_mul_small<C>(B, run, lo - 1, bits);
+  if (alpha > 1) {  // warp-uniform
+    xyzz_mul_small<C>(B, tri, alpha, 32 - __clz(alpha));
+    tri = B;
+  }
+  const uint32_t kmax = alpha * (NB - 1) + beta;
+  xyzz_mul_small<C>(B, run, alpha * lo + beta, 32 - __clz(kmax | 1u));
   xyzz_add_ni<C>(tri, tri, B);
   store_xyzz<C>(out + (size_t)gid * XW, tri);
 }

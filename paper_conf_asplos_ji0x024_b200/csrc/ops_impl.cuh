@@ -82,7 +82,10 @@ struct Ops final : CurveOps {
     s.nwin = num_windows(C::LAMBDA, c);
     s.pre = pre;
     s.nset = pre ? 1 : s.nwin;
-    s.NB = (1u << (c - 1)) + 1;
+    s.split_G = o.split_G;
+    s.split_g = o.split_g;
+    s.c_arg = c | ((o.split_G - 1) << 8) | (o.split_g << 16);
+    s.NB = (1u << (c - 1)) / (uint32_t)o.split_G + 1;
     s.F = (size_t)s.nset * s.NB;
     s.ntiles = cdiv(s.F, SCAN_TILE);
     // a3 variant: the staged three-level sort for large entry counts, the binned two-level
@@ -90,8 +93,8 @@ struct Ops final : CurveOps {
     const size_t Mmax0 = s.n * (size_t)s.nwin;
     s.sort_mode = o.sort ? o.sort : (Mmax0 >= ((size_t)1 << 21) ? 3 : 2);
     s.shift = 0;
-    while (s.shift < 13 && (size_t)s.nset * ((((size_t)1 << (c - 1)) >> s.shift) + 1) > 13000) s.shift++;
-    s.nbin = (uint32_t)((((size_t)1 << (c - 1)) >> s.shift) + 1);
+    while (s.shift < 13 && (size_t)s.nset * (((size_t)(s.NB - 1) >> s.shift) + 1) > 13000) s.shift++;
+    s.nbin = (uint32_t)(((size_t)(s.NB - 1) >> s.shift) + 1);
     s.FB = (uint32_t)s.nset * s.nbin;
     s.ntiles_bin = cdiv(s.FB, SCAN_TILE);
     CK(cudaFuncSetAttribute(k_bin_count<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(s.FB * 4)));
@@ -120,7 +123,7 @@ struct Ops final : CurveOps {
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps2, k_bucket_segments<C>, 128, 0));
     if (bps2 < 1) bps2 = 1;
     const size_t resident2 = (size_t)sms * bps2 * 128;
-    const size_t nb = s.NB - 1;
+    const size_t nb = s.NB;  // local buckets 0..NB-1 (bucket 0 is empty without the f1 split)
     // one segment per resident thread (full occupancy, no tail wave); >= 4 buckets each
     uint32_t seg = o.seg > 0 ? (uint32_t)o.seg : (uint32_t)std::max<size_t>(4, cdiv((size_t)s.nset * nb, resident2));
     s.seg = seg;
@@ -149,7 +152,7 @@ struct Ops final : CurveOps {
       // b1, b2 <= 9 per partition pass
       int KB = 1;
       while (((size_t)1 << KB) < s.F) KB++;
-      int b3 = (int)std::lround(std::log2(8192.0 * (double)s.F / (double)std::max<size_t>(Mmax, 1)));
+      int b3 = (int)std::lround(std::log2(8192.0 * (double)s.F / (double)std::max<size_t>(Mmax / (size_t)s.split_G, 1)));
       b3 = std::max(1, std::min(b3, 12));
       b3 = std::min(b3, KB);
       if (KB - b3 > 18) b3 = KB - 18;
@@ -196,7 +199,7 @@ struct Ops final : CurveOps {
       const int sh1 = s.s3_b2 + s.s3_b3;
       CK(cudaMemsetAsync(s.s3Count, 0, NC1 * sizeof(uint32_t), st));
       if (n) {
-        k_s3_count1<C><<<(unsigned)cdiv(n, S3_THREADS * 16), S3_THREADS, 0, st>>>(scal, n, s.c, s.nwin, ws, sh1, NC1,
+        k_s3_count1<C><<<(unsigned)cdiv(n, S3_THREADS * 16), S3_THREADS, 0, st>>>(scal, n, s.c_arg, s.nwin, ws, sh1, NC1,
                                                                                s.s3Count, s.err);
         launches++;
       }
@@ -207,7 +210,7 @@ struct Ops final : CurveOps {
       launches += 3;
       const uint32_t tp = (uint32_t)std::max(1, S3_TILE / s.nwin);
       if (n) {
-        k_s3_part1<C><<<(unsigned)cdiv(n, tp), S3_THREADS, 2 * S3_TILE * 4, st>>>(scal, n, s.c, s.nwin, ws, istride, sh1,
+        k_s3_part1<C><<<(unsigned)cdiv(n, tp), S3_THREADS, 2 * S3_TILE * 4, st>>>(scal, n, s.c_arg, s.nwin, ws, istride, sh1,
                                                                                 NC1, tp, s.s3Cursor, s.s3k1, s.s3v1);
         launches++;
       }
@@ -229,7 +232,7 @@ struct Ops final : CurveOps {
       CK(cudaMemsetAsync(s.binCount, 0, s.FB * sizeof(uint32_t), st));
       const unsigned tiles = (unsigned)cdiv(std::max<size_t>(n, 1), BIN_TILE);
       if (n) {
-        k_bin_count<C><<<tiles, BIN_THREADS, s.FB * 4, st>>>(scal, n, s.c, s.nwin, s.shift, s.FB, wsb, s.binCount, s.err);
+        k_bin_count<C><<<tiles, BIN_THREADS, s.FB * 4, st>>>(scal, n, s.c_arg, s.nwin, s.shift, s.FB, wsb, s.binCount, s.err);
         launches++;
       }
       k_scan_reduce<<<(unsigned)s.ntiles_bin, SCAN_THREADS, 0, st>>>(s.binCount, s.FB, s.tiles);
@@ -237,7 +240,7 @@ struct Ops final : CurveOps {
       k_scan_apply<<<(unsigned)s.ntiles_bin, SCAN_THREADS, 0, st>>>(s.binCount, s.FB, s.tiles, s.binOff, s.binCursor);
       launches += 3;
       if (n) {
-        k_bin_scatter<C><<<tiles, BIN_THREADS, 2 * s.FB * 4, st>>>(scal, n, s.c, s.nwin, s.shift, s.FB, wsb, istride,
+        k_bin_scatter<C><<<tiles, BIN_THREADS, 2 * s.FB * 4, st>>>(scal, n, s.c_arg, s.nwin, s.shift, s.FB, wsb, istride,
                                                                   s.binCursor, s.binIdx, s.binFine);
         launches++;
       }
@@ -250,7 +253,7 @@ struct Ops final : CurveOps {
     } else {
       CK(cudaMemsetAsync(s.counts, 0, s.F * sizeof(uint32_t), st));
       if (n) {
-        k_digit_counts<C><<<(unsigned)cdiv(n, 256), 256, 0, st>>>(scal, n, s.c, s.nwin, ws, s.counts, s.err);
+        k_digit_counts<C><<<(unsigned)cdiv(n, 256), 256, 0, st>>>(scal, n, s.c_arg, s.nwin, ws, s.counts, s.err);
         launches++;
       }
       k_scan_reduce<<<(unsigned)s.ntiles, SCAN_THREADS, 0, st>>>(s.counts, s.F, s.tiles);
@@ -258,7 +261,7 @@ struct Ops final : CurveOps {
       k_scan_apply<<<(unsigned)s.ntiles, SCAN_THREADS, 0, st>>>(s.counts, s.F, s.tiles, s.goff, s.cursor);
       launches += 3;
       if (n) {
-        k_digit_scatter<C><<<(unsigned)cdiv(n, 256), 256, 0, st>>>(scal, n, s.c, s.nwin, ws, istride, s.cursor, s.sorted);
+        k_digit_scatter<C><<<(unsigned)cdiv(n, 256), 256, 0, st>>>(scal, n, s.c_arg, s.nwin, ws, istride, s.cursor, s.sorted);
         launches++;
       }
     }
@@ -284,7 +287,8 @@ struct Ops final : CurveOps {
     if (timed) CK(cudaEventRecord(s.ev[EV_FIX], st));
     // a5: bucket reduce
     const uint32_t total = (uint32_t)s.nset * s.nseg;
-    k_bucket_segments<C><<<(unsigned)cdiv(total, 128), 128, 0, st>>>(s.buckets, s.goff, s.nset, s.NB, s.seg, s.nseg, s.segA);
+    k_bucket_segments<C><<<(unsigned)cdiv(total, 128), 128, 0, st>>>(s.buckets, s.goff, s.nset, s.NB, s.seg, s.nseg,
+                                                                      (uint32_t)s.split_G, (uint32_t)s.split_g, s.segA);
     launches++;
     uint32_t nin = s.nseg;
     uint32_t* src = s.segA;

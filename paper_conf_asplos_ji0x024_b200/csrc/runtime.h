@@ -52,7 +52,9 @@ struct Shard {
   int c = 0, nwin = 0;
   int pre = 0;         // precomputed window table in use (f3): one bucket set for all windows
   int nset = 0;        // bucket sets: nwin (pre = 0) or 1 (pre = 1)
-  uint32_t NB = 0;     // buckets per set incl. bucket 0 = 2^(c-1) + 1
+  uint32_t NB = 0;     // (local) buckets per set incl. bucket 0 = 2^(c-1)/G + 1
+  int split_G = 1, split_g = 0;  // f1 bucket split: part g of G
+  int c_arg = 0;       // c | (G-1) << 8 | g << 16 for the digit kernels (for_each_digit)
   size_t F = 0;        // flat buckets = nset * NB
   uint32_t acc_threads = 0, slice = 0;
   uint32_t seg = 0, nseg = 0;
@@ -90,6 +92,7 @@ struct Options {
   int sort = 0;  // a3 variant: 0 auto, 1 direct global atomics (ablation), 2 two-level binned,
                  // 3 three-level staged (sort3.cuh)
   int pre = 2;   // f3 precomputation: 0 off, 1 on, 2 auto (on when the table fits in memory)
+  int split_G = 1, split_g = 0;  // f1: this context sums only buckets |d| = G*q + g
 };
 
 // Per-curve kernels behind a virtual interface (one instance per curve, curve_*.cu).

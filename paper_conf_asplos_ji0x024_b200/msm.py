@@ -25,6 +25,8 @@ OPT_ACC_THREADS = 2
 OPT_SEG_LEN = 3
 OPT_SORT = 4
 OPT_PRECOMPUTE = 5
+OPT_SPLIT_PARTS = 6
+OPT_SPLIT_INDEX = 7
 OPT_NWIN = 101
 OPT_NONEMPTY = 102
 OPT_NSETS = 103

@@ -327,3 +327,69 @@ def test_degenerate_top_window(lib, cbits):
     ctx.set_option(lib.OPT_WINDOW_BITS, cbits)
     assert ctx.run(synth.ints_to_words(ks, 8)) == closed(name, ks, es)
     ctx.close()
+
+
+@pytest.mark.parametrize("name", ["bn254", "bls12_381", "mnt4_753"])
+@pytest.mark.parametrize("pre", [0, 1])
+def test_bucket_split_parity(lib, name, pre):
+    """f1 bucket split: G contexts over ALL points, context g summing only
+    the buckets |d| = G*q + g.  Each part's partial (affine through msm_finalize) equals the
+    oracle's part (stages.bucket_split_partial, computed from the definition), and the G
+    partials finalize to the closed form.  Ragged n, G not dividing 2^(c-1), O points and
+    duplicates (doubling inside a part)."""
+    c = CURVES[name]
+    n = 45 if name == "mnt4_753" else 131
+    Ps, es, _, _ = progression(name, n, 41)
+    Ps = list(Ps)
+    Ps[2] = None
+    Ps[7] = Ps[6]
+    ks = synth.words_to_ints(synth.scalars(c.r, n, 43))
+    ks[6] = ks[7]
+    e = [0 if P is None else x for P, x in zip(Ps, es)]
+    e[7] = es[6]
+    sw = synth.ints_to_words(ks, S_W[name])
+    pw = lib.partial_words(name)
+    for cbits, G in ((5, 3), (7, 2), (6, 5)):
+        parts = np.zeros(G * pw, dtype=np.uint32)
+        for g in range(G):
+            ctx = lib.Context(name, points_to_words(Ps, name), n=n)
+            ctx.set_option(lib.OPT_PRECOMPUTE, pre)
+            ctx.set_option(lib.OPT_WINDOW_BITS, cbits)
+            ctx.set_option(lib.OPT_SPLIT_PARTS, G)
+            ctx.set_option(lib.OPT_SPLIT_INDEX, g)
+            assert ctx.get_option(lib.OPT_SPLIT_PARTS) == G and ctx.get_option(lib.OPT_SPLIT_INDEX) == g
+            ctx.run_partial(sw, parts[g * pw:(g + 1) * pw])
+            ctx.close()
+            want_g = ec.to_output(stages.bucket_split_partial(ks, Ps, cbits, c, G, g, bool(pre)))
+            assert lib.finalize(name, parts[g * pw:(g + 1) * pw], 1) == want_g, (cbits, G, g)
+        assert lib.finalize(name, parts, G) == closed(name, ks, e), (cbits, G)
+
+
+def test_bucket_split_large_balanced(lib):
+    """f1 at a size that uses the staged sort and many segments: BLS12-381, n = 2^16, auto c
+    with the f3 table, G = 4 parts finalize to the closed form, and the interleaved
+    assignment keeps every part's entry count within 2 % of the mean."""
+    name = "bls12_381"
+    c = CURVES[name]
+    n = 1 << 16
+    e0, d = synth.point_seeds(c.r, 77)
+    import torch
+    pts = torch.empty((n, 2 * L32[name]), dtype=torch.int32, device="cuda")
+    lib.gen_points(name, e0, d, n, pts)
+    ks = synth.scalars_range(c.r, 0, n, 78)
+    es_sum = sum(k * ((e0 + i * d) % c.r) for i, k in enumerate(synth.words_to_ints(ks))) % c.r
+    want = ec.to_output(ec.mul(es_sum, c.G, c))
+    G = 4
+    pw = lib.partial_words(name)
+    parts = np.zeros(G * pw, dtype=np.uint32)
+    entries = []
+    for g in range(G):
+        ctx = lib.Context(name, pts, n=n)
+        ctx.set_option(lib.OPT_SPLIT_PARTS, G)
+        ctx.set_option(lib.OPT_SPLIT_INDEX, g)
+        ctx.run_partial(ks, parts[g * pw:(g + 1) * pw])
+        entries.append(ctx.stats()["entries"])
+        ctx.close()
+    assert lib.finalize(name, parts, G) == want
+    mean = sum(entries) / G
+    assert max(abs(x - mean) for x in entries) < 0.02 * mean, entries

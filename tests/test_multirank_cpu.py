@@ -82,3 +82,50 @@ def test_two_rank_gather_and_split_invariance():
     assert res[0] == "ok", res
     assert res[1] is True
     assert res[2] == [(0, 18), (18, 19)]
+
+
+def _worker_buckets(rank, world, port, q):
+    """f1 bucket split: every rank holds ALL points and scalars and owns the
+    buckets b = |d| with b mod world = rank; the oracle's part stands in for the GPU partial."""
+    os.environ["MASTER_ADDR"] = "127.0.0.1"
+    os.environ["MASTER_PORT"] = str(port)
+    dist.init_process_group("gloo", rank=rank, world_size=world)
+    try:
+        import synth
+        from oracle import ec, msm as omsm, points as opoints, stages
+        from oracle.curves import CURVES
+        c = CURVES["bn254"]
+        n = 23
+        ks = synth.words_to_ints(synth.scalars_range(c.r, 0, n, 12))
+        e0, d = synth.point_seeds(c.r, 13)
+        Ps = opoints.progression_points(e0, d, n, c)
+        x, y = ec.to_output(stages.bucket_split_partial(ks, Ps, 5, c, world, rank, pre=False))
+        words = torch.tensor([(x >> (32 * i)) & 0xFFFFFFFF for i in range(8)] +
+                             [(y >> (32 * i)) & 0xFFFFFFFF for i in range(8)], dtype=torch.int64).to(torch.int32)
+        allp = gather_partials(words)
+        if rank == 0:
+            tot = None
+            for r_ in range(world):
+                w = allp[r_].to(torch.int64) & 0xFFFFFFFF
+                px = sum(int(w[i]) << (32 * i) for i in range(8))
+                py = sum(int(w[8 + i]) << (32 * i) for i in range(8))
+                tot = ec.add(tot, None if (px, py) == (0, 0) else (px, py), c)
+            q.put(("ok", tot == omsm.msm_naive(ks, Ps, c), None))
+    except Exception as ex:  # pragma: no cover
+        q.put(("err", repr(ex), None))
+    finally:
+        dist.destroy_process_group()
+
+
+def test_two_rank_bucket_split():
+    ctx = mp.get_context("spawn")
+    q = ctx.Queue()
+    port = _free_port()
+    ps = [ctx.Process(target=_worker_buckets, args=(r, 2, port, q)) for r in range(2)]
+    for p in ps:
+        p.start()
+    res = q.get(timeout=240)
+    for p in ps:
+        p.join(timeout=60)
+    assert res[0] == "ok", res
+    assert res[1] is True

@@ -116,3 +116,31 @@ def test_precomputed_route(c):
                 acc = ec.add(acc, ec.mul(pow(2, j * cc), Bw[j][b], c) if Bw[j][b] else None, c)
             assert Bp[b] == acc, b
         assert stages.msm_precomputed(ks, Ps, cc, c) == want
+
+
+@pytest.mark.parametrize("c", [CURVES["bn254"], CURVES["bls12_381"]], ids=lambda c: c.name)
+def test_bucket_split_parts_sum_to_msm(c):
+    """f1 bucket split: the G parts' partials add up to the closed form for
+    several G (incl. G not dividing 2^(c-1)) with and without the f3 table, and one part
+    (G = 1) is the whole MSM.  A wrong weight, a dropped residue class or a part counted
+    twice breaks the sum."""
+    n = 20
+    e0, d = synth.point_seeds(c.r, 6)
+    Ps = points.progression_points(e0, d, n, c)
+    es = points.progression_scalars(e0, d, n, c)
+    ks = synth.words_to_ints(synth.scalars(c.r, n, 17))
+    ks[3] = c.r - 1
+    ks[4] = 1
+    want = msm.msm_closed_form(ks, es, c)
+    for pre in (False, True):
+        for cc, G in ((5, 2), (5, 3), (6, 5), (4, 8)):
+            parts = [stages.bucket_split_partial(ks, Ps, cc, c, G, g, pre) for g in range(G)]
+            tot = None
+            for P in parts:
+                tot = ec.add(tot, P, c)
+            assert tot == want, (pre, cc, G)
+        assert stages.bucket_split_partial(ks, Ps, 5, c, 1, 0, pre) == want
+    # a part is not the whole: with G = 2 both halves are generically non-trivial and differ
+    h0 = stages.bucket_split_partial(ks, Ps, 5, c, 2, 0)
+    h1 = stages.bucket_split_partial(ks, Ps, 5, c, 2, 1)
+    assert h0 != h1 and h0 is not None and h1 is not None
