@@ -144,6 +144,27 @@ int msm_run_partial(msm_context* ctx, const uint32_t* scalars, uint32_t* partial
  */
 int msm_finalize(int curve, const uint32_t* partials, int count, uint32_t* result);
 
+/*
+ * Pipelined MSMs on one context (ngpus == 1), for a stream of MSMs over the same points
+ * (the proving workload): msm_submit enqueues one MSM — H2D copy of its
+ * scalars on a copy stream, the a2..a7 kernels on the compute stream — and returns a
+ * ticket (>= 0) without waiting.  The copy of MSM t+1's scalars starts as soon as MSM t's
+ * sort stage has consumed the device scalar buffer, so it overlaps MSM t's accumulation.
+ * msm_wait(ctx, ticket, result) blocks until MSM `ticket` is done and writes its canonical
+ * affine result (2*L32 host words).  At most MSM_MAX_INFLIGHT tickets may be outstanding
+ * (submitted, not yet waited for); tickets must be waited for in submission order.
+ * `scalars`: host (pinned memory copies at full PCIe rate) or device; the caller keeps the
+ * buffer valid and unmodified until msm_wait of that ticket returns.
+ * Errors: msm_submit returns MSM_ERR_ARG (NULL, ngpus > 1, too many outstanding) or a CUDA
+ * code; msm_wait returns MSM_ERR_ARG (not the oldest outstanding ticket), MSM_ERR_SCALAR
+ * (some k_i >= r: no result written; later tickets are unaffected) or a CUDA code.
+ * Statistics (msm_get_stats) describe the most recently waited-for MSM when it was also
+ * the most recently submitted one.
+ */
+#define MSM_MAX_INFLIGHT 2
+long msm_submit(msm_context* ctx, const uint32_t* scalars);
+int msm_wait(msm_context* ctx, long ticket, uint32_t* result);
+
 int msm_set_option(msm_context* ctx, int key, long value);
 long msm_get_option(msm_context* ctx, int key);
 int msm_get_stats(const msm_context* ctx, msm_stats* out);

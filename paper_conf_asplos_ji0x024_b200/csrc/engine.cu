@@ -32,6 +32,13 @@ struct msm_context {
   msm_stats stats{};
   CurveOps* ops = nullptr;
   int launches = 0;
+  // pipelined submit/wait (single shard): ring of MSM_MAX_INFLIGHT result slots
+  cudaStream_t copy_stream = nullptr;
+  cudaEvent_t ev_copied = nullptr;
+  cudaEvent_t ev_done[MSM_MAX_INFLIGHT] = {};
+  uint32_t* d_result[MSM_MAX_INFLIGHT] = {};
+  uint32_t* h_result = nullptr;  // pinned [MSM_MAX_INFLIGHT][2*L32 + 1] (last word: error flags)
+  long next_ticket = 0, next_wait = 0;
 };
 
 namespace {
@@ -380,6 +387,18 @@ msm_context* msm_context_create(int curve, const uint32_t* points, size_t n, int
 
 void msm_context_destroy(msm_context* ctx) {
   if (!ctx) return;
+  if (ctx->copy_stream) {
+    cudaSetDevice(ctx->shards[0].dev);
+    cudaStreamSynchronize(ctx->shards[0].stream);
+    cudaStreamSynchronize(ctx->copy_stream);
+    cudaStreamDestroy(ctx->copy_stream);
+    cudaEventDestroy(ctx->ev_copied);
+    for (int q = 0; q < MSM_MAX_INFLIGHT; q++) {
+      cudaEventDestroy(ctx->ev_done[q]);
+      dfree(ctx->d_result[q]);
+    }
+    cudaFreeHost(ctx->h_result);
+  }
   for (auto& s : ctx->shards) destroy_shard(ctx->ops, s);
   delete ctx;
 }
@@ -419,6 +438,65 @@ int msm_run_partial(msm_context* ctx, const uint32_t* scalars, uint32_t* partial
     } else {
       CK(cudaMemcpy(partial, s0.partial, ctx->ops->XW() * 4, cudaMemcpyDeviceToHost));
     }
+    return MSM_OK;
+  });
+}
+
+long msm_submit(msm_context* ctx, const uint32_t* scalars) {
+  if (!ctx || (ctx->n && !scalars) || ctx->shards.size() != 1) return MSM_ERR_ARG;
+  if (ctx->next_ticket - ctx->next_wait >= MSM_MAX_INFLIGHT) return MSM_ERR_ARG;
+  const int rc = guarded([&]() -> int {
+    Shard& s = ctx->shards[0];
+    const int L32 = ctx->ops->L32();
+    CK(cudaSetDevice(s.dev));
+    if (!ctx->copy_stream) {
+      CK(cudaStreamCreateWithFlags(&ctx->copy_stream, cudaStreamNonBlocking));
+      CK(cudaEventCreateWithFlags(&ctx->ev_copied, cudaEventDisableTiming));
+      for (int q = 0; q < MSM_MAX_INFLIGHT; q++) {
+        CK(cudaEventCreateWithFlags(&ctx->ev_done[q], cudaEventDisableTiming));
+        dalloc(&ctx->d_result[q], 2 * L32);
+      }
+      CK(cudaMallocHost((void**)&ctx->h_result, MSM_MAX_INFLIGHT * (2 * L32 + 1) * 4));
+    }
+    const int q = (int)(ctx->next_ticket % MSM_MAX_INFLIGHT);
+    // copy stream: wait until the previous MSM's sort has consumed s.scal (EV_SORT is
+    // re-recorded by every pipeline, so this waits on the latest one), then H2D
+    CK(cudaStreamWaitEvent(ctx->copy_stream, s.ev[EV_SORT], 0));
+    const size_t bytes = s.n * (size_t)ctx->ops->S() * 4;
+    if (bytes) CK(cudaMemcpyAsync(s.scal, scalars + s.off * ctx->ops->S(), bytes, cudaMemcpyDefault, ctx->copy_stream));
+    CK(cudaEventRecord(ctx->ev_copied, ctx->copy_stream));
+    // compute stream: a2..a6 on the staged scalars, then finalise into result slot q
+    CK(cudaStreamWaitEvent(s.stream, ctx->ev_copied, 0));
+    CK(cudaEventRecord(s.ev[EV_START], s.stream));
+    CK(cudaMemsetAsync(s.err, 0, 4, s.stream));
+    ctx->launches = ctx->ops->enqueue_pipeline(s, s.scal, true);
+    ctx->ops->enqueue_finalize(s.partial, 1, ctx->d_result[q], s.stream);
+    ctx->launches++;
+    CK(cudaEventRecord(s.ev[EV_END], s.stream));
+    uint32_t* h = ctx->h_result + q * (2 * L32 + 1);
+    CK(cudaMemcpyAsync(h, ctx->d_result[q], 2 * L32 * 4, cudaMemcpyDeviceToHost, s.stream));
+    CK(cudaMemcpyAsync(h + 2 * L32, s.err, 4, cudaMemcpyDeviceToHost, s.stream));
+    CK(cudaEventRecord(ctx->ev_done[q], s.stream));
+    return MSM_OK;
+  });
+  return rc == MSM_OK ? ctx->next_ticket++ : (long)rc;
+}
+
+int msm_wait(msm_context* ctx, long ticket, uint32_t* result) {
+  if (!ctx || !result || ticket != ctx->next_wait || ticket >= ctx->next_ticket) return MSM_ERR_ARG;
+  return guarded([&]() -> int {
+    Shard& s = ctx->shards[0];
+    const int L32 = ctx->ops->L32();
+    const int q = (int)(ticket % MSM_MAX_INFLIGHT);
+    CK(cudaSetDevice(s.dev));
+    CK(cudaEventSynchronize(ctx->ev_done[q]));
+    ctx->next_wait++;
+    if (ticket + 1 == ctx->next_ticket) collect_stats(ctx);
+    const uint32_t* h = ctx->h_result + q * (2 * L32 + 1);
+    const uint32_t e = h[2 * L32];
+    if (e & 4u) return MSM_ERR_SCALAR;
+    if (e & 3u) return MSM_ERR_POINT;
+    std::memcpy(result, h, 2 * L32 * 4);
     return MSM_OK;
   });
 }

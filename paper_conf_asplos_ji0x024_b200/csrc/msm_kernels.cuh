@@ -644,7 +644,14 @@ __global__ void __launch_bounds__(128, MSM_ACC_MINB) k_accumulate(const uint32_t
   bool ok = point_for_entry<C>(x, y, pts, __ldg(sorted + e0));
   acc_start<C>(acc, x, y, ok);
   int32_t my_carry = -1;
-#if MSM_ACC_PREFETCH
+#if MSM_ACC_PREFETCH == 2
+  // A/B: two PACCs ahead (indices read three ahead)
+  uint32_t ent1 = e0 + 1 < e1 ? __ldg(sorted + e0 + 1) : 0u;
+  uint32_t ent2 = e0 + 2 < e1 ? __ldg(sorted + e0 + 2) : 0u;
+  uint32_t ent3 = e0 + 3 < e1 ? __ldg(sorted + e0 + 3) : 0u;
+  if (e0 + 1 < e1) prefetch_point<C>(pts, ent1);
+  if (e0 + 2 < e1) prefetch_point<C>(pts, ent2);
+#elif MSM_ACC_PREFETCH
   // the gathered point of entry e+1 is prefetched into L1 one PACC ahead (its index
   // read two ahead), so the random 8L-byte gather does not stall the next iteration
   uint32_t ent1 = e0 + 1 < e1 ? __ldg(sorted + e0 + 1) : 0u;
@@ -652,7 +659,13 @@ __global__ void __launch_bounds__(128, MSM_ACC_MINB) k_accumulate(const uint32_t
   if (e0 + 1 < e1) prefetch_point<C>(pts, ent1);
 #endif
   for (uint32_t e = e0 + 1; e < e1; e++) {
-#if MSM_ACC_PREFETCH
+#if MSM_ACC_PREFETCH == 2
+    const uint32_t ent = ent1;
+    ent1 = ent2;
+    ent2 = ent3;
+    if (e + 2 < e1) prefetch_point<C>(pts, ent2);
+    if (e + 3 < e1) ent3 = __ldg(sorted + e + 3);
+#elif MSM_ACC_PREFETCH
     const uint32_t ent = ent1;
     ent1 = ent2;
     if (e + 1 < e1) prefetch_point<C>(pts, ent1);

@@ -72,6 +72,7 @@ def lib() -> ctypes.CDLL:
         "msm_partial_words": (i, [i]), "msm_device_count": (i, []),
         "msm_context_create": (P, [i, P, sz, i]), "msm_context_destroy": (None, [P]),
         "msm_run": (i, [P, P, P]), "msm_run_partial": (i, [P, P, P]), "msm_finalize": (i, [i, P, i, P]),
+        "msm_submit": (ctypes.c_long, [P, P]), "msm_wait": (i, [P, ctypes.c_long, P]),
         "msm_set_option": (i, [P, i, ctypes.c_long]), "msm_get_option": (ctypes.c_long, [P, i]),
         "msm_get_stats": (i, [P, ctypes.POINTER(Stats)]), "msm_get_stream": (P, [P, i]),
         "msm_last_error": (i, []), "msm_error_string": (ctypes.c_char_p, [i]),
@@ -187,6 +188,30 @@ class Context:
     def run(self, scalars):
         """Q = sum k_i P_i as affine ints (x, y); O -> (0, 0)."""
         return point_from_words(self.run_words(scalars), self.L32)
+
+    def submit(self, scalars) -> int:
+        """Pipelined MSM (msm_submit): enqueue and return a ticket; the scalar buffer is kept
+        alive here until wait(ticket)."""
+        sp, keep = _ptr(scalars, words=self.n * self.S) if self.n else (None, None)
+        t = lib().msm_submit(self._h, sp)
+        if t < 0:
+            raise MSMError(int(t), "msm_submit")
+        if not hasattr(self, "_inflight"):
+            self._inflight = {}
+        self._inflight[t] = keep
+        return t
+
+    def wait_words(self, ticket: int, out=None) -> np.ndarray:
+        res = np.zeros(2 * self.L32, dtype=np.uint32) if out is None else out
+        try:
+            _check(lib().msm_wait(self._h, ticket, ctypes.c_void_p(res.ctypes.data)), "msm_wait")
+        finally:
+            getattr(self, "_inflight", {}).pop(ticket, None)
+        return res
+
+    def wait(self, ticket: int):
+        """Result of a submitted MSM as affine ints (x, y)."""
+        return point_from_words(self.wait_words(ticket), self.L32)
 
     def run_partial(self, scalars, out):
         sp, keep = _ptr(scalars, words=self.n * self.S) if self.n else (None, None)

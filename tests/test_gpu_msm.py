@@ -393,3 +393,40 @@ def test_bucket_split_large_balanced(lib):
     assert lib.finalize(name, parts, G) == want
     mean = sum(entries) / G
     assert max(abs(x - mean) for x in entries) < 0.02 * mean, entries
+
+
+@pytest.mark.parametrize("name", ["bn254", "bls12_381", "mnt4_753"])
+def test_pipelined_submit_wait(lib, name):
+    """msm_submit / msm_wait: interleaved submissions (the next MSM's H2D overlaps the
+    current one) give each MSM's own closed-form result; a scalar >= r fails only its own
+    ticket; over-submission and out-of-order waits are rejected; the context stays usable
+    and agrees with msm_run."""
+    c = CURVES[name]
+    n = 700 if name != "mnt4_753" else 90
+    Ps, es, _, _ = progression(name, n, 61)
+    ctx = lib.Context(name, points_to_words(Ps, name), n=n)
+    sets = [synth.words_to_ints(synth.scalars(c.r, n, 70 + t)) for t in range(5)]
+    bad = list(sets[3])
+    bad[n // 2] = c.r  # k >= r
+    words = [synth.ints_to_words(k, S_W[name]) for k in sets]
+    words[3] = synth.ints_to_words(bad, S_W[name])
+    t0 = ctx.submit(words[0])
+    t1 = ctx.submit(words[1])
+    with pytest.raises(lib.MSMError):
+        ctx.submit(words[2])           # MSM_MAX_INFLIGHT = 2 outstanding
+    with pytest.raises(lib.MSMError):
+        ctx.wait(t1)                   # not the oldest outstanding ticket
+    assert ctx.wait(t0) == closed(name, sets[0], es)
+    t2 = ctx.submit(words[2])
+    assert ctx.wait(t1) == closed(name, sets[1], es)
+    t3 = ctx.submit(words[3])
+    t4 = ctx.submit(words[4])
+    assert ctx.wait(t2) == closed(name, sets[2], es)
+    with pytest.raises(lib.MSMError) as ei:
+        ctx.wait(t3)
+    assert ei.value.code == -7         # MSM_ERR_SCALAR, this ticket only
+    assert ctx.wait(t4) == closed(name, sets[4], es)
+    assert ctx.run(words[1]) == closed(name, sets[1], es)
+    t5 = ctx.submit(words[0])
+    assert ctx.wait(t5) == closed(name, sets[0], es)
+    ctx.close()

@@ -1,8 +1,10 @@
-timeout 1200 python -m pytest tests -m gpu -x -q > gpurun_out/gputests.log 2>&1
+timeout 1500 python -m pytest tests -m gpu -x -q > gpurun_out/gputests.log 2>&1
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > gpurun_out/smoke.log 2>&1
 timeout 600 python bench.py --check > gpurun_out/bench.log 2>&1
-for sp in buckets points; do
-  MSM_BENCH_SHARE_DEVICE=1 timeout 600 python -m torch.distributed.run --nnodes=1 --nproc-per-node 2 --master-addr 127.0.0.1 --master-port 29511 \
-    bench.py --gpus 2 --log2n 22 --split $sp --check --steps 2 --no-cpu-baseline > gpurun_out/share2_$sp.log 2>&1
-done
-for so in 1 3; do timeout 600 python bench.py --log2n 24 --sort $so --steps 3 --no-e2e --no-cpu-baseline --check 2>/dev/null | tail -1 >> gpurun_out/sort_ablation.jsonl; done
+python tools/ab.py --log2n 24 base pf2 > gpurun_out/ab_pf2.jsonl 2>&1
+python tools/ab.py --log2n 26 --steps 2 base pf2 >> gpurun_out/ab_pf2.jsonl 2>&1
+OUT=gpurun_out/prof_sort NOLAUNCH=1 KERNELS="k_s3_count1 k_s3_part1 k_s3_part2 k_s3_part3" bash tools/profile_round.sh
+timeout 900 ncu --set full --import-source on --clock-control none -k regex:k_accumulate -s 3 -c 1 -o gpurun_out/acc_src -f python bench.py --log2n 22 --steps 1 --warmup 3 --no-e2e --no-cpu-baseline > gpurun_out/acc_src.log 2>&1
+ncu -i gpurun_out/acc_src.ncu-rep --page source --csv --print-source sass > gpurun_out/acc_src_sass.csv 2>&1
+gzip -f gpurun_out/acc_src_sass.csv
+rm -f gpurun_out/acc_src.ncu-rep
