@@ -246,20 +246,6 @@ DEVI bool scalar_in_range(const ScalarReg<C>& k) {
   return lt;
 }
 
-// bits [bit, bit + c) of k, c <= 31
-template <class C>
-DEVI uint32_t scalar_bits(const ScalarReg<C>& k, int bit, int c) {
-  const int wi = bit >> 5, sh = bit & 31;
-  uint32_t lo = 0, hi = 0;
-#pragma unroll
-  for (int q = 0; q < C::S; q++) {
-    if (q == wi) lo = k.w[q];
-    if (q == wi + 1) hi = k.w[q];
-  }
-  uint64_t v = ((uint64_t)hi << 32) | lo;
-  return (uint32_t)(v >> sh) & ((1u << c) - 1u);
-}
-
 // Walks the windows of one scalar, calling f(j, bucket, negative) for non-zero digits.
 // cp = c | (G - 1) << 8 | g << 16 packs the f1 bucket split ("splits the
 // buckets into GPUs-per-window parts"): with G > 1 only digits |d| = G*q + g are emitted,
@@ -268,10 +254,18 @@ template <class C, class F>
 DEVI void for_each_digit(const ScalarReg<C>& k, int cp, int nwin, F&& f) {
   const int c = cp & 0xff;
   const uint32_t G = ((uint32_t)(cp >> 8) & 0xffu) + 1u, g = (uint32_t)(cp >> 16) & 0xffu;
-  const uint32_t half = 1u << (c - 1);
+  const uint32_t half = 1u << (c - 1), cmask = (1u << c) - 1u;
+  // the scalar is consumed by funnel shifts (S SHF per window; c <= 24 < 32), instead of
+  // selecting the window's words with runtime indices (~4S ALU ops per window)
+  uint32_t w[C::S];
+#pragma unroll
+  for (int q = 0; q < C::S; q++) w[q] = k.w[q];
   uint32_t carry = 0;
   for (int j = 0; j < nwin; j++) {
-    uint32_t d = scalar_bits<C>(k, j * c, c) + carry;
+    uint32_t d = (w[0] & cmask) + carry;
+#pragma unroll
+    for (int q = 0; q < C::S - 1; q++) w[q] = __funnelshift_r(w[q], w[q + 1], c);
+    w[C::S - 1] >>= c;
     bool neg = false;
     if (j < nwin - 1 && d > half) {
       d = (1u << c) - d;
@@ -580,7 +574,7 @@ DEVI bool point_for_entry(uint32_t* x, uint32_t* y, const uint32_t* __restrict__
 }
 
 #ifndef MSM_ACC_PREFETCH
-#define MSM_ACC_PREFETCH 1
+#define MSM_ACC_PREFETCH 3  // next point gather: 3 registers (L <= 13), 2/1 L1 prefetch, 0 none
 #endif
 #ifndef MSM_ACC_PADD
 #define MSM_ACC_PADD 0  // f4 ablation: PADD (Alg. 1) with Z = 1 operand instead of PACC (Alg. 4)
@@ -644,36 +638,57 @@ __global__ void __launch_bounds__(128, MSM_ACC_MINB) k_accumulate(const uint32_t
   bool ok = point_for_entry<C>(x, y, pts, __ldg(sorted + e0));
   acc_start<C>(acc, x, y, ok);
   int32_t my_carry = -1;
-#if MSM_ACC_PREFETCH == 2
-  // A/B: two PACCs ahead (indices read three ahead)
-  uint32_t ent1 = e0 + 1 < e1 ? __ldg(sorted + e0 + 1) : 0u;
-  uint32_t ent2 = e0 + 2 < e1 ? __ldg(sorted + e0 + 2) : 0u;
-  uint32_t ent3 = e0 + 3 < e1 ? __ldg(sorted + e0 + 3) : 0u;
-  if (e0 + 1 < e1) prefetch_point<C>(pts, ent1);
-  if (e0 + 2 < e1) prefetch_point<C>(pts, ent2);
-#elif MSM_ACC_PREFETCH
-  // the gathered point of entry e+1 is prefetched into L1 one PACC ahead (its index
-  // read two ahead), so the random 8L-byte gather does not stall the next iteration
-  uint32_t ent1 = e0 + 1 < e1 ? __ldg(sorted + e0 + 1) : 0u;
-  uint32_t ent2 = e0 + 2 < e1 ? __ldg(sorted + e0 + 2) : 0u;
-  if (e0 + 1 < e1) prefetch_point<C>(pts, ent1);
-#endif
+  // Gather of the next entry's stored point (PF, A/B-able with MSM_ACC_PREFETCH):
+  //   3  into REGISTERS one PACC ahead (index read two ahead) — default for L <= 13.  The
+  //      first use of a gathered point was the top stall site of the kernel (ncu source
+  //      view: the zero test of y waiting on the gather, ~4 % of samples) even with an L1
+  //      prefetch, because the L1 hit latency itself sat on the critical path; 26 more
+  //      registers keep 8 warps/SM.  MNT4-753 (L = 27, already at 255 registers) keeps 1.
+  //   2  L1 prefetch two PACCs ahead;  1  L1 prefetch one PACC ahead;  0  none.
+  constexpr int PF = (MSM_ACC_PREFETCH == 3 && C::L > 13) ? 1 : MSM_ACC_PREFETCH;
+  uint32_t nx[C::L], ny[C::L];
+  uint32_t ent1 = 0, ent2 = 0, ent3 = 0;
+  if constexpr (PF > 0) {
+    ent1 = e0 + 1 < e1 ? __ldg(sorted + e0 + 1) : 0u;
+    ent2 = e0 + 2 < e1 ? __ldg(sorted + e0 + 2) : 0u;
+    if constexpr (PF == 3) {
+      if (e0 + 1 < e1) load_point<C>(nx, ny, pts, ent1 & ~SIGN_BIT);
+    } else {
+      if (e0 + 1 < e1) prefetch_point<C>(pts, ent1);
+    }
+    if constexpr (PF == 2) {
+      ent3 = e0 + 3 < e1 ? __ldg(sorted + e0 + 3) : 0u;
+      if (e0 + 2 < e1) prefetch_point<C>(pts, ent2);
+    }
+  }
   for (uint32_t e = e0 + 1; e < e1; e++) {
-#if MSM_ACC_PREFETCH == 2
-    const uint32_t ent = ent1;
-    ent1 = ent2;
-    ent2 = ent3;
-    if (e + 2 < e1) prefetch_point<C>(pts, ent2);
-    if (e + 3 < e1) ent3 = __ldg(sorted + e + 3);
-#elif MSM_ACC_PREFETCH
-    const uint32_t ent = ent1;
-    ent1 = ent2;
-    if (e + 1 < e1) prefetch_point<C>(pts, ent1);
-    if (e + 2 < e1) ent2 = __ldg(sorted + e + 2);
-#else
-    const uint32_t ent = __ldg(sorted + e);
-#endif
-    ok = point_for_entry<C>(x, y, pts, ent);
+    uint32_t ent;
+    if constexpr (PF == 3) {
+      ent = ent1;
+      ent1 = ent2;
+      fcopy<C>(x, nx);
+      fcopy<C>(y, ny);
+      if (e + 1 < e1) load_point<C>(nx, ny, pts, ent1 & ~SIGN_BIT);
+      if (e + 2 < e1) ent2 = __ldg(sorted + e + 2);
+      ok = !fis_zero<C, 2>(y);
+      if (ok && (ent & SIGN_BIT)) fneg<C, 2>(y, y);
+    } else {
+      if constexpr (PF == 2) {
+        ent = ent1;
+        ent1 = ent2;
+        ent2 = ent3;
+        if (e + 2 < e1) prefetch_point<C>(pts, ent2);
+        if (e + 3 < e1) ent3 = __ldg(sorted + e + 3);
+      } else if constexpr (PF == 1) {
+        ent = ent1;
+        ent1 = ent2;
+        if (e + 1 < e1) prefetch_point<C>(pts, ent1);
+        if (e + 2 < e1) ent2 = __ldg(sorted + e + 2);
+      } else {
+        ent = __ldg(sorted + e);
+      }
+      ok = point_for_entry<C>(x, y, pts, ent);
+    }
     if (e == end) {
       if (head) { store_xyzz<C>(carry_pts + (size_t)t * XW, acc); my_carry = (int32_t)f; head = false; }
       else store_xyzz<C>(buckets + (size_t)f * XW, acc);

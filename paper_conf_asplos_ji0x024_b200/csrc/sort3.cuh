@@ -25,6 +25,41 @@ constexpr int S3_CAP = 12288;        // largest sub-bin P3 sorts in shared memor
 constexpr int S3_MAXB = 512;         // max bins per partition pass (b1, b2 <= 9)
 constexpr int S3_MAXFINE = 4096;     // max buckets per sub-bin (b3 <= 12)
 
+// Entry loops over [e0, e1) with stride blockDim.x, S3_U loads in flight per thread: the
+// P2/P3 passes were global-load-latency bound (ncu: long_scoreboard ~35-49 stalls per
+// issue, 14-17 % issue) with one key load outstanding per thread.
+constexpr int S3_U = 8;
+template <class F>
+__device__ __forceinline__ void s3_for_keys(const uint32_t* __restrict__ keys, uint32_t e0, uint32_t e1, F&& f) {
+  for (uint32_t eb = e0 + threadIdx.x; eb < e1; eb += S3_U * blockDim.x) {
+    uint32_t k[S3_U];
+#pragma unroll
+    for (int u = 0; u < S3_U; u++) {
+      const uint32_t e = eb + u * blockDim.x;
+      k[u] = e < e1 ? __ldg(keys + e) : 0u;
+    }
+#pragma unroll
+    for (int u = 0; u < S3_U; u++)
+      if (eb + u * blockDim.x < e1) f(k[u]);
+  }
+}
+template <class F>
+__device__ __forceinline__ void s3_for_entries(const uint32_t* __restrict__ keys, const uint32_t* __restrict__ vals,
+                                               uint32_t e0, uint32_t e1, F&& f) {
+  for (uint32_t eb = e0 + threadIdx.x; eb < e1; eb += S3_U * blockDim.x) {
+    uint32_t k[S3_U], v[S3_U];
+#pragma unroll
+    for (int u = 0; u < S3_U; u++) {
+      const uint32_t e = eb + u * blockDim.x;
+      k[u] = e < e1 ? __ldg(keys + e) : 0u;
+      v[u] = e < e1 ? __ldg(vals + e) : 0u;
+    }
+#pragma unroll
+    for (int u = 0; u < S3_U; u++)
+      if (eb + u * blockDim.x < e1) f(k[u], v[u]);
+  }
+}
+
 // exclusive scan of cnt[0..N) in place (N <= blockDim.x * per-thread chunk); returns total
 __device__ __forceinline__ uint32_t s3_block_scan(uint32_t* cnt, uint32_t N, uint32_t* warp_sums) {
   const uint32_t per = (N + blockDim.x - 1) / blockDim.x;
@@ -157,7 +192,7 @@ static __global__ void __launch_bounds__(S3_THREADS) k_s3_count2(const uint32_t*
   const uint32_t mask = NC2 - 1;
   for (uint32_t i = threadIdx.x; i < NC2; i += blockDim.x) hist[i] = 0;
   __syncthreads();
-  for (uint32_t e = e0 + threadIdx.x; e < e1; e += blockDim.x) atomicAdd(hist + ((__ldg(keys + e) >> sh2) & mask), 1u);
+  s3_for_keys(keys, e0, e1, [&](uint32_t f) { atomicAdd(hist + ((f >> sh2) & mask), 1u); });
   __syncthreads();
   for (uint32_t i = threadIdx.x; i < NC2; i += blockDim.x)
     if (hist[i]) atomicAdd(subCount + (size_t)bin * NC2 + i, hist[i]);
@@ -180,7 +215,7 @@ static __global__ void __launch_bounds__(S3_THREADS) k_s3_part2(const uint32_t* 
   const uint32_t mask = NC2 - 1;
   for (uint32_t i = threadIdx.x; i < NC2; i += blockDim.x) cur[i] = 0;
   __syncthreads();
-  for (uint32_t e = e0 + threadIdx.x; e < e1; e += blockDim.x) atomicAdd(cur + ((__ldg(keys + e) >> sh2) & mask), 1u);
+  s3_for_keys(keys, e0, e1, [&](uint32_t f) { atomicAdd(cur + ((f >> sh2) & mask), 1u); });
   __syncthreads();
   for (uint32_t i = threadIdx.x; i < NC2; i += blockDim.x) {
     const uint32_t h = cur[i];
@@ -191,12 +226,11 @@ static __global__ void __launch_bounds__(S3_THREADS) k_s3_part2(const uint32_t* 
   const uint32_t E = s3_block_scan(loc, NC2, warp_sums);
   for (uint32_t i = threadIdx.x; i < NC2; i += blockDim.x) cur[i] = loc[i];
   __syncthreads();
-  for (uint32_t e = e0 + threadIdx.x; e < e1; e += blockDim.x) {
-    const uint32_t f = __ldg(keys + e);
+  s3_for_entries(keys, vals, e0, e1, [&](uint32_t f, uint32_t v) {
     const uint32_t pos = atomicAdd(cur + ((f >> sh2) & mask), 1u);
     skey[pos] = f;
-    sval[pos] = __ldg(vals + e);
-  }
+    sval[pos] = v;
+  });
   __syncthreads();
   for (uint32_t p = threadIdx.x; p < E; p += blockDim.x) {
     const uint32_t f = skey[p], sb = (f >> sh2) & mask;
@@ -220,7 +254,7 @@ static __global__ void __launch_bounds__(256) k_s3_part3(const uint32_t* __restr
   const uint32_t nf = 1u << b3, fmask = nf - 1, fbase = q << b3;
   for (uint32_t i = threadIdx.x; i < nf; i += blockDim.x) cnt[i] = 0;
   __syncthreads();
-  for (uint32_t e = e0 + threadIdx.x; e < e1; e += blockDim.x) atomicAdd(cnt + (__ldg(keys2 + e) & fmask), 1u);
+  s3_for_keys(keys2, e0, e1, [&](uint32_t f) { atomicAdd(cnt + (f & fmask), 1u); });
   __syncthreads();
   s3_block_scan(cnt, nf, warp_sums);
   for (uint32_t i = threadIdx.x; i < nf; i += blockDim.x)
@@ -228,10 +262,7 @@ static __global__ void __launch_bounds__(256) k_s3_part3(const uint32_t* __restr
   __syncthreads();
   const uint32_t len = e1 - e0;
   if (len <= (uint32_t)S3_CAP) {
-    for (uint32_t e = e0 + threadIdx.x; e < e1; e += blockDim.x) {
-      const uint32_t f = __ldg(keys2 + e);
-      sval[atomicAdd(cnt + (f & fmask), 1u)] = __ldg(vals2 + e);
-    }
+    s3_for_entries(keys2, vals2, e0, e1, [&](uint32_t f, uint32_t v) { sval[atomicAdd(cnt + (f & fmask), 1u)] = v; });
     __syncthreads();
     for (uint32_t p = threadIdx.x; p < len; p += blockDim.x) sorted[e0 + p] = sval[p];
   } else {  // oversized sub-bin (skewed scalars): scatter straight to global

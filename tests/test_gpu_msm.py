@@ -420,8 +420,8 @@ def test_pipelined_submit_wait(lib, name):
     t2 = ctx.submit(words[2])
     assert ctx.wait(t1) == closed(name, sets[1], es)
     t3 = ctx.submit(words[3])
-    t4 = ctx.submit(words[4])
     assert ctx.wait(t2) == closed(name, sets[2], es)
+    t4 = ctx.submit(words[4])
     with pytest.raises(lib.MSMError) as ei:
         ctx.wait(t3)
     assert ei.value.code == -7         # MSM_ERR_SCALAR, this ticket only
