@@ -21,6 +21,10 @@ typedef unsigned long long u64;
 
 #define DEVI __device__ __forceinline__
 
+#ifndef MSM_FMUL2_LAT
+#define MSM_FMUL2_LAT 0  // A/B: fmul2 columns with the a*b chain split in two (6 chains per warp)
+#endif
+
 #ifndef MSM_FSQR_AS_MUL
 #define MSM_FSQR_AS_MUL 0
 #endif
@@ -171,8 +175,8 @@ template <class C, bool SQR, int K>
 DEVI void fmul2_cols(uint32_t* r1, const uint32_t* a1, const uint32_t* b1, const uint32_t* a21, uint32_t* m1,
                      u64 cA1, u64 cM1, uint32_t* r2, const uint32_t* a2, const uint32_t* b2, const uint32_t* a22,
                      uint32_t* m2, u64 cA2, u64 cM2) {
-  fmul_step<C, SQR, false, K>(r1, a1, b1, a21, m1, cA1, cM1);
-  fmul_step<C, SQR, false, K>(r2, a2, b2, a22, m2, cA2, cM2);
+  fmul_step<C, SQR, MSM_FMUL2_LAT != 0, K>(r1, a1, b1, a21, m1, cA1, cM1);
+  fmul_step<C, SQR, MSM_FMUL2_LAT != 0, K>(r2, a2, b2, a22, m2, cA2, cM2);
   if constexpr (K + 1 < 2 * C::L - 1)
     fmul2_cols<C, SQR, K + 1>(r1, a1, b1, a21, m1, cA1, cM1, r2, a2, b2, a22, m2, cA2, cM2);
 }

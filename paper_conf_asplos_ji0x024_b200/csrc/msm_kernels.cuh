@@ -579,6 +579,13 @@ DEVI bool point_for_entry(uint32_t* x, uint32_t* y, const uint32_t* __restrict__
 #ifndef MSM_ACC_PADD
 #define MSM_ACC_PADD 0  // f4 ablation: PADD (Alg. 1) with Z = 1 operand instead of PACC (Alg. 4)
 #endif
+#ifndef MSM_ACC_SYNC
+#define MSM_ACC_SYNC 1  // k_accumulate_sync (256-thread blocks in per-iteration lockstep) for L <= 13
+#endif
+#ifndef MSM_SEG_SYNC
+#define MSM_SEG_SYNC 0  // A/B: k_bucket_segments with 256-thread blocks in per-bucket lockstep
+#endif
+constexpr int SEG_NT = MSM_SEG_SYNC ? 256 : 128;
 #ifndef MSM_ACC_SMEM
 #define MSM_ACC_SMEM 0  // A/B: k_accumulate_smem (operands in shared-memory slots, one fmul2 body)
 #endif
@@ -714,6 +721,77 @@ __global__ void __launch_bounds__(128, MSM_ACC_MINB) k_accumulate(const uint32_t
   if (head) { store_xyzz<C>(carry_pts + (size_t)t * XW, acc); my_carry = (int32_t)f; }
   else store_xyzz<C>(buckets + (size_t)f * XW, acc);
   carry_f[t] = my_carry;
+}
+
+// ---------------------------------------------------------------------------------------
+// a4 variant (MSM_ACC_SYNC, A/B): 256-thread blocks, one per SM (2 warps per scheduler as
+// in k_accumulate), with a block barrier at the top of every PACC iteration so the two
+// warps of each scheduler walk the ~90 KB straight-line PACC code in lockstep and share
+// instruction fetches (ncu: no_instruction is 17 % of k_accumulate's stall samples, spread
+// evenly over the straight-line code).  Every thread runs the same number of iterations
+// (the uniform slice length); threads without work only take part in the barriers.
+constexpr int ACC_SYNC_NT = 256;
+template <class C>
+__global__ void __launch_bounds__(ACC_SYNC_NT, 1) k_accumulate_sync(const uint32_t* __restrict__ pts, const uint32_t* __restrict__ sorted,
+                                                    const uint32_t* __restrict__ goff, uint32_t F,
+                                                    uint32_t* __restrict__ buckets, uint32_t* __restrict__ carry_pts,
+                                                    int32_t* __restrict__ carry_f, uint32_t nthreads,
+                                                    uint32_t* __restrict__ nlong) {
+  constexpr int XW = Layout<C>::XW;
+  const uint32_t t = blockIdx.x * blockDim.x + threadIdx.x;
+  if (t == 0) *nlong = 0;
+  const uint32_t M = __ldg(goff + F);
+  const uint32_t slice = M ? (M + nthreads - 1) / nthreads : 1u;
+  const uint64_t e0l = (uint64_t)t * slice;
+  const bool active = t < nthreads && e0l < M;
+  if (t < nthreads && !active) carry_f[t] = -1;
+  const uint32_t e0 = active ? (uint32_t)e0l : 0u;
+  const uint32_t e1 = active ? (uint32_t)(e0l + slice < (uint64_t)M ? e0l + slice : (uint64_t)M) : 0u;
+  uint32_t f = 0, end = 0;
+  bool head = false, ok = false;
+  Xyzz<C> acc;
+  uint32_t x[C::L], y[C::L], nx[C::L], ny[C::L];
+  uint32_t ent1 = 0, ent2 = 0;
+  int32_t my_carry = -1;
+  if (active) {
+    f = find_bucket(goff, F, e0);
+    end = __ldg(goff + f + 1);
+    head = __ldg(goff + f) < e0;
+    ok = point_for_entry<C>(x, y, pts, __ldg(sorted + e0));
+    acc_start<C>(acc, x, y, ok);
+    ent1 = e0 + 1 < e1 ? __ldg(sorted + e0 + 1) : 0u;
+    ent2 = e0 + 2 < e1 ? __ldg(sorted + e0 + 2) : 0u;
+    if (e0 + 1 < e1) load_point<C>(nx, ny, pts, ent1 & ~SIGN_BIT);
+  }
+  for (uint32_t q = 1; q < slice; q++) {
+    __syncthreads();
+    const uint32_t e = e0 + q;
+    if (!active || e >= e1) continue;
+    const uint32_t ent = ent1;
+    ent1 = ent2;
+    fcopy<C>(x, nx);
+    fcopy<C>(y, ny);
+    if (e + 1 < e1) load_point<C>(nx, ny, pts, ent1 & ~SIGN_BIT);
+    if (e + 2 < e1) ent2 = __ldg(sorted + e + 2);
+    ok = !fis_zero<C, 2>(y);
+    if (ok && (ent & SIGN_BIT)) fneg<C, 2>(y, y);
+    if (e == end) {
+      if (head) { store_xyzz<C>(carry_pts + (size_t)t * XW, acc); my_carry = (int32_t)f; head = false; }
+      else store_xyzz<C>(buckets + (size_t)f * XW, acc);
+      do { f++; end = __ldg(goff + f + 1); } while (end <= e);
+      acc_start<C>(acc, x, y, ok);
+    } else if (ok) {
+      if (xyzz_acc_hot<C>(acc, x, y)) {
+        Xyzz<C> T = acc;
+        xyzz_dbl<C>(acc, T);
+      }
+    }
+  }
+  if (active) {
+    if (head) { store_xyzz<C>(carry_pts + (size_t)t * XW, acc); my_carry = (int32_t)f; }
+    else store_xyzz<C>(buckets + (size_t)f * XW, acc);
+    carry_f[t] = my_carry;
+  }
 }
 
 // ---------------------------------------------------------------------------------------
@@ -1079,23 +1157,26 @@ DEVI void xyzz_mul_small(Xyzz<C>& R, const Xyzz<C>& A, uint32_t k, int bits) {
 // and the segment's share of W_j = sum_q (alpha q + beta) B_q is
 //   alpha*tri + (alpha*lo + beta)*run.
 template <class C>
-__global__ void __launch_bounds__(128, MSM_SEG_MINB) k_bucket_segments(const uint32_t* __restrict__ buckets, const uint32_t* __restrict__ goff,
+__global__ void __launch_bounds__(SEG_NT, MSM_SEG_SYNC ? 1 : MSM_SEG_MINB) k_bucket_segments(const uint32_t* __restrict__ buckets, const uint32_t* __restrict__ goff,
                                                          int nwin, uint32_t NB, uint32_t seg, uint32_t nseg,
                                                          uint32_t alpha, uint32_t beta,
                                                          uint32_t* __restrict__ out) {
   constexpr int XW = Layout<C>::XW;
   const uint32_t gid = blockIdx.x * blockDim.x + threadIdx.x;
-  if (gid >= (uint32_t)nwin * nseg) return;
-  const uint32_t j = gid / nseg, t = gid % nseg;
+  // MSM_SEG_SYNC: lanes past the last segment stay (as O segments) for the block barriers
+  const bool live = gid < (uint32_t)nwin * nseg;
+  if (!MSM_SEG_SYNC && !live) return;
+  const uint32_t j = live ? gid / nseg : 0u, t = live ? gid % nseg : 0u;
   const uint32_t lo = t * seg;
   Xyzz<C> run, tri, B;
   xyzz_set_zero<C>(run);
   xyzz_set_zero<C>(tri);
   // uniform trip count `seg`; buckets past NB - 1 and empty buckets contribute O
   for (uint32_t q = seg; q-- > 0;) {
+    if (MSM_SEG_SYNC) __syncthreads();  // lockstep: shared instruction fetch (see k_accumulate_sync)
     const uint32_t b = lo + q;
     const size_t f = (size_t)j * NB + b;
-    const bool ne = b < NB && __ldg(goff + f + 1) != __ldg(goff + f);
+    const bool ne = live && b < NB && __ldg(goff + f + 1) != __ldg(goff + f);
     if (ne) load_xyzz<C>(B, buckets + f * XW);
     else xyzz_set_zero<C>(B);
     xyzz_add_hot<C>(run, run, B);
@@ -1108,7 +1189,7 @@ __global__ void __launch_bounds__(128, MSM_SEG_MINB) k_bucket_segments(const uin
   const uint32_t kmax = alpha * (NB - 1) + beta;
   xyzz_mul_small<C>(B, run, alpha * lo + beta, 32 - __clz(kmax | 1u));
   xyzz_add_ni<C>(tri, tri, B);
-  store_xyzz<C>(out + (size_t)gid * XW, tri);
+  if (live) store_xyzz<C>(out + (size_t)gid * XW, tri);
 }
 
 // out[j*nout + g] = sum of in[j*nin + g*group .. + group)   (per window)

@@ -13,6 +13,9 @@ using namespace msmk;
 
 template <class C>
 struct Ops final : CurveOps {
+  // k_accumulate_sync (lockstep blocks, register-prefetched gathers) for L <= 13; MNT4-753
+  // keeps k_accumulate (255 registers already; no room for the prefetched point)
+  static constexpr bool kAccSync = MSM_ACC_SYNC != 0 && C::L <= 13;
   static constexpr int XW_ = Layout<C>::XW;
   static constexpr int PW_ = Layout<C>::PW;
   int L32() const override { return C::L32; }
@@ -109,7 +112,12 @@ struct Ops final : CurveOps {
     CK(cudaFuncSetAttribute(k_accumulate_smem<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, acc_smem));
     CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_accumulate_smem<C>, 128, acc_smem));
 #else
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_accumulate<C>, 128, 0));
+    if constexpr (kAccSync) {
+      CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_accumulate_sync<C>, ACC_SYNC_NT, 0));
+      bps *= ACC_SYNC_NT / 128;  // in units of 128 threads below
+    } else {
+      CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, k_accumulate<C>, 128, 0));
+    }
 #endif
     if (bps < 1) bps = 1;
     const size_t resident = (size_t)sms * bps * 128;
@@ -120,7 +128,8 @@ struct Ops final : CurveOps {
     s.acc_threads = (uint32_t)std::max<size_t>(1, cdiv(Mmax, s.slice));
     // bucket-reduce segments
     int bps2 = 0;
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps2, k_bucket_segments<C>, 128, 0));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps2, k_bucket_segments<C>, SEG_NT, 0));
+    bps2 *= SEG_NT / 128;  // in units of 128 threads below
     if (bps2 < 1) bps2 = 1;
     const size_t resident2 = (size_t)sms * bps2 * 128;
     const size_t nb = s.NB;  // local buckets 0..NB-1 (bucket 0 is empty without the f1 split)
@@ -271,7 +280,12 @@ struct Ops final : CurveOps {
 #if MSM_ACC_SMEM
     k_accumulate_smem<C><<<(unsigned)cdiv(s.acc_threads, 128), 128, ACC_SLOTS * C::L * ACC_NT * 4, st>>>(pts, s.sorted, s.goff, (uint32_t)s.F,
 #else
-    k_accumulate<C><<<(unsigned)cdiv(s.acc_threads, 128), 128, 0, st>>>(pts, s.sorted, s.goff, (uint32_t)s.F,
+    if constexpr (kAccSync)
+      k_accumulate_sync<C><<<(unsigned)cdiv(s.acc_threads, ACC_SYNC_NT), ACC_SYNC_NT, 0, st>>>(pts, s.sorted, s.goff, (uint32_t)s.F,
+                                                                        s.buckets, s.carry_pts, s.carry_f, s.acc_threads,
+                                                                        s.nlong);
+    else
+      k_accumulate<C><<<(unsigned)cdiv(s.acc_threads, 128), 128, 0, st>>>(pts, s.sorted, s.goff, (uint32_t)s.F,
 #endif
                                                                         s.buckets, s.carry_pts, s.carry_f, s.acc_threads,
                                                                         s.nlong);
@@ -287,7 +301,7 @@ struct Ops final : CurveOps {
     if (timed) CK(cudaEventRecord(s.ev[EV_FIX], st));
     // a5: bucket reduce
     const uint32_t total = (uint32_t)s.nset * s.nseg;
-    k_bucket_segments<C><<<(unsigned)cdiv(total, 128), 128, 0, st>>>(s.buckets, s.goff, s.nset, s.NB, s.seg, s.nseg,
+    k_bucket_segments<C><<<(unsigned)cdiv(total, SEG_NT), SEG_NT, 0, st>>>(s.buckets, s.goff, s.nset, s.NB, s.seg, s.nseg,
                                                                       (uint32_t)s.split_G, (uint32_t)s.split_g, s.segA);
     launches++;
     uint32_t nin = s.nseg;
