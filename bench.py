@@ -408,7 +408,7 @@ def main():
                           "peak_basis": "MEASURED_PEAKS.json hbm_gbs (copy bandwidth)"},
         "stages_ms": {k: round(v, 3) for k, v in st.items() if k.endswith("_ms") and k != "table_ms"},
         "latency_ms": {"mean": ms, "min": min(times), "max": max(times)},
-        "roofline": {"kernel": "k_accumulate", "bound": "alu", "achieved": achieved / 1e12, "peak": peak_slots / 1e12,
+        "roofline": {"kernel": "k_accumulate_sync" if L <= 13 else "k_accumulate", "bound": "alu", "achieved": achieved / 1e12, "peak": peak_slots / 1e12,
                      "unit": "T IMAD-pipe slots/s", "frac": achieved / peak_slots, "traffic": ncu_traffic(curve, args.log2n),
                      "work": f"{pacc} PACC x (8 mul x {imad_slots_per_mult(L)} + 2 sqr x {imad_slots_per_sqr(L)}) IMAD slots",
                      "peak_basis": f"148 SM x 64 IMAD slots/clk x {sm_max} MHz (clocks.max.sm); IMAD.WIDE = 2 slots (measured)",

@@ -582,6 +582,9 @@ DEVI bool point_for_entry(uint32_t* x, uint32_t* y, const uint32_t* __restrict__
 #ifndef MSM_ACC_SYNC
 #define MSM_ACC_SYNC 1  // k_accumulate_sync (256-thread blocks in per-iteration lockstep) for L <= 13
 #endif
+#ifndef MSM_ACC_SYNC_ALL
+#define MSM_ACC_SYNC_ALL 0  // A/B: lockstep accumulation for MNT4-753 too (L1 prefetch there)
+#endif
 #ifndef MSM_SEG_SYNC
 #define MSM_SEG_SYNC 0  // A/B: k_bucket_segments with 256-thread blocks in per-bucket lockstep
 #endif
@@ -753,6 +756,9 @@ __global__ void __launch_bounds__(ACC_SYNC_NT, 1) k_accumulate_sync(const uint32
   uint32_t x[C::L], y[C::L], nx[C::L], ny[C::L];
   uint32_t ent1 = 0, ent2 = 0;
   int32_t my_carry = -1;
+  // next point into registers one PACC ahead (L <= 13), or an L1 prefetch for MNT4-753
+  // whose 255 registers leave no room for it
+  constexpr bool REGPF = C::L <= 13;
   if (active) {
     f = find_bucket(goff, F, e0);
     end = __ldg(goff + f + 1);
@@ -761,7 +767,11 @@ __global__ void __launch_bounds__(ACC_SYNC_NT, 1) k_accumulate_sync(const uint32
     acc_start<C>(acc, x, y, ok);
     ent1 = e0 + 1 < e1 ? __ldg(sorted + e0 + 1) : 0u;
     ent2 = e0 + 2 < e1 ? __ldg(sorted + e0 + 2) : 0u;
-    if (e0 + 1 < e1) load_point<C>(nx, ny, pts, ent1 & ~SIGN_BIT);
+    if constexpr (REGPF) {
+      if (e0 + 1 < e1) load_point<C>(nx, ny, pts, ent1 & ~SIGN_BIT);
+    } else {
+      if (e0 + 1 < e1) prefetch_point<C>(pts, ent1);
+    }
   }
   for (uint32_t q = 1; q < slice; q++) {
     __syncthreads();
@@ -769,12 +779,18 @@ __global__ void __launch_bounds__(ACC_SYNC_NT, 1) k_accumulate_sync(const uint32
     if (!active || e >= e1) continue;
     const uint32_t ent = ent1;
     ent1 = ent2;
-    fcopy<C>(x, nx);
-    fcopy<C>(y, ny);
-    if (e + 1 < e1) load_point<C>(nx, ny, pts, ent1 & ~SIGN_BIT);
-    if (e + 2 < e1) ent2 = __ldg(sorted + e + 2);
-    ok = !fis_zero<C, 2>(y);
-    if (ok && (ent & SIGN_BIT)) fneg<C, 2>(y, y);
+    if constexpr (REGPF) {
+      fcopy<C>(x, nx);
+      fcopy<C>(y, ny);
+      if (e + 1 < e1) load_point<C>(nx, ny, pts, ent1 & ~SIGN_BIT);
+      if (e + 2 < e1) ent2 = __ldg(sorted + e + 2);
+      ok = !fis_zero<C, 2>(y);
+      if (ok && (ent & SIGN_BIT)) fneg<C, 2>(y, y);
+    } else {
+      if (e + 1 < e1) prefetch_point<C>(pts, ent1);
+      if (e + 2 < e1) ent2 = __ldg(sorted + e + 2);
+      ok = point_for_entry<C>(x, y, pts, ent);
+    }
     if (e == end) {
       if (head) { store_xyzz<C>(carry_pts + (size_t)t * XW, acc); my_carry = (int32_t)f; head = false; }
       else store_xyzz<C>(buckets + (size_t)f * XW, acc);

@@ -15,7 +15,7 @@ template <class C>
 struct Ops final : CurveOps {
   // k_accumulate_sync (lockstep blocks, register-prefetched gathers) for L <= 13; MNT4-753
   // keeps k_accumulate (255 registers already; no room for the prefetched point)
-  static constexpr bool kAccSync = MSM_ACC_SYNC != 0 && C::L <= 13;
+  static constexpr bool kAccSync = MSM_ACC_SYNC != 0 && (C::L <= 13 || MSM_ACC_SYNC_ALL != 0);
   static constexpr int XW_ = Layout<C>::XW;
   static constexpr int PW_ = Layout<C>::PW;
   int L32() const override { return C::L32; }
