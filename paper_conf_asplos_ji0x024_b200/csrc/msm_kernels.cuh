@@ -733,7 +733,10 @@ __global__ void __launch_bounds__(128, MSM_ACC_MINB) k_accumulate(const uint32_t
 // instruction fetches (ncu: no_instruction is 17 % of k_accumulate's stall samples, spread
 // evenly over the straight-line code).  Every thread runs the same number of iterations
 // (the uniform slice length); threads without work only take part in the barriers.
-constexpr int ACC_SYNC_NT = 256;
+#ifndef MSM_ACC_SYNC_NT
+#define MSM_ACC_SYNC_NT 256  // A/B: 384 = 3 warps per scheduler (<= 168 registers)
+#endif
+constexpr int ACC_SYNC_NT = MSM_ACC_SYNC_NT;
 template <class C>
 __global__ void __launch_bounds__(ACC_SYNC_NT, 1) k_accumulate_sync(const uint32_t* __restrict__ pts, const uint32_t* __restrict__ sorted,
                                                     const uint32_t* __restrict__ goff, uint32_t F,
