@@ -184,8 +184,9 @@ int msm_gen_points(int curve, const uint32_t* e0, const uint32_t* delta, size_t 
 
 /*
  * Test-only entry points (host buffers; run on the current device; synchronous).
- *   msm_debug_field: op 0 mul, 1 sqr, 2 add, 3 sub, 4 inv, 5 neg on n canonical
- *     elements a[i], b[i] (L32 words each); out[i] canonical.
+ *   msm_debug_field: op 0 mul, 1 sqr, 2 add, 3 sub, 4 inv (Fermat), 5 neg, 6 inv (binary
+ *     extended Euclid, the one the final normalisation uses) on n canonical elements
+ *     a[i], b[i] (L32 words each); out[i] canonical (inv of 0 is 0 for op 6).
  *   msm_debug_ec: op 0 acc (P + Q via Alg. 4 with P in XYZZ scaled by z1), 1 add (Alg. 1,
  *     both scaled by z1/z2), 2 dbl; P, Q affine (2*L32 words, (0,0) = O); z: 2*L32 words
  *     per element (z1, z2 non-zero canonical); out: affine.

@@ -617,7 +617,7 @@ int msm_gen_points(int curve, const uint32_t* e0, const uint32_t* delta, size_t 
 int msm_debug_field(int curve, int op, const uint32_t* a, const uint32_t* b, size_t n, uint32_t* out) {
   CurveOps* ops = ops_for(curve);
   if (!ops) return MSM_ERR_CURVE;
-  if (!a || !b || !out || op < 0 || op > 5) return MSM_ERR_ARG;
+  if (!a || !b || !out || op < 0 || op > 6) return MSM_ERR_ARG;
   return guarded([&]() -> int {
     ops->debug_field(op, a, b, n, out);
     return MSM_OK;

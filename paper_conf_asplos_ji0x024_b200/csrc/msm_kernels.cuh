@@ -1339,7 +1339,7 @@ __global__ void __launch_bounds__(128) k_gen_points(const uint32_t* __restrict__
 
 // ---------------------------------------------------------------------------------------
 // debug kernels for the field / EC layers (tests only)
-enum { DBG_MUL = 0, DBG_SQR = 1, DBG_ADD = 2, DBG_SUB = 3, DBG_INV = 4, DBG_NEG = 5 };
+enum { DBG_MUL = 0, DBG_SQR = 1, DBG_ADD = 2, DBG_SUB = 3, DBG_INV = 4, DBG_NEG = 5, DBG_INV_BGCD = 6 };
 
 template <class C>
 __global__ void k_debug_field(int op, const uint32_t* __restrict__ a, const uint32_t* __restrict__ b, size_t n,
@@ -1358,6 +1358,7 @@ __global__ void k_debug_field(int op, const uint32_t* __restrict__ a, const uint
     case DBG_ADD: fadd<C>(r, x, y); break;
     case DBG_SUB: fsub<C, 2>(r, x, y); break;
     case DBG_INV: finv<C>(r, x); break;
+    case DBG_INV_BGCD: finv_bgcd<C>(r, x); break;
     default: fneg<C, 2>(r, x); break;
   }
   ffrom_mont<C>(r, r);

@@ -55,6 +55,12 @@ def test_field_ops(msm, name):
     a2 = np.stack([to_words(v, w) for v in nz])
     got = msm.debug_field(name, 4, a2, a2)
     assert all(from_words(got[i]) == pow(nz[i], -1, p) for i in range(len(nz)))
+    # binary-GCD inversion (the final normalisation's): every non-zero edge value and
+    # random values; 0 maps to 0 (no inverse) instead of looping
+    got = msm.debug_field(name, 6, a2, a2)
+    assert all(from_words(got[i]) == pow(nz[i], -1, p) for i in range(len(nz)))
+    z = np.zeros((4, w), dtype=np.uint32)
+    assert not msm.debug_field(name, 6, z, z).any()
 
 
 def _z_words(c, n, seed):
