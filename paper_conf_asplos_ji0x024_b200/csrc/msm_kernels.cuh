@@ -19,6 +19,9 @@ constexpr uint32_t SIGN_BIT = 0x80000000u;
 #ifndef MSM_ACC_MINB
 #define MSM_ACC_MINB 1  // min resident 128-thread blocks per SM for k_accumulate (register cap)
 #endif
+#ifndef MSM_SUM_WARP
+#define MSM_SUM_WARP 1  // k_sum_groups as a warp shuffle tree per group (0: one thread per group)
+#endif
 #ifndef MSM_SEG_MINB
 #define MSM_SEG_MINB 1
 #endif
@@ -1228,6 +1231,36 @@ __global__ void __launch_bounds__(128) k_sum_groups(const uint32_t* __restrict__
     xyzz_add_ni<C>(s, s, b);
   }
   store_xyzz<C>(out + (size_t)gid * XW, s);
+}
+
+// The same sums with one warp per group (MSM_SUM_WARP, default): lane q loads input q of the
+// group and a five-step shuffle tree adds them, so each level of the tree costs 5 serial
+// PADDs instead of 32.  Every lane runs every add (lanes past the live half add copies of
+// themselves; only lane 0's sum is stored), so the out-of-line PADD is called convergently.
+template <class C>
+__global__ void __launch_bounds__(128) k_sum_groups_warp(const uint32_t* __restrict__ in, uint32_t nin, uint32_t group,
+                                                         uint32_t nout, int nwin, uint32_t* __restrict__ out) {
+  constexpr int XW = Layout<C>::XW, L = C::L;
+  const uint32_t gid = (blockIdx.x * blockDim.x + threadIdx.x) >> 5, lane = threadIdx.x & 31;
+  if (gid >= (uint32_t)nwin * nout) return;  // warp-uniform
+  const uint32_t j = gid / nout, g = gid % nout;
+  Xyzz<C> s, b;
+  const uint32_t i = g * group + lane;
+  if (lane < group && i < nin) load_xyzz<C>(s, in + ((size_t)j * nin + i) * XW);
+  else xyzz_set_zero<C>(s);
+#pragma unroll 1
+  for (int off = 16; off >= 1; off >>= 1) {
+#pragma unroll
+    for (int k = 0; k < L; k++) {
+      b.X[k] = __shfl_down_sync(0xffffffffu, s.X[k], off);
+      b.Y[k] = __shfl_down_sync(0xffffffffu, s.Y[k], off);
+      b.ZZ[k] = __shfl_down_sync(0xffffffffu, s.ZZ[k], off);
+      b.ZZZ[k] = __shfl_down_sync(0xffffffffu, s.ZZZ[k], off);
+    }
+    if (lane + off >= 32) xyzz_set_zero<C>(b);
+    xyzz_add_ni<C>(s, s, b);
+  }
+  if (lane == 0) store_xyzz<C>(out + (size_t)gid * XW, s);
 }
 
 // ---------------------------------------------------------------------------------------

@@ -311,7 +311,11 @@ struct Ops final : CurveOps {
       const uint32_t group = nin > 32 ? 32 : nin;
       const uint32_t nout = (uint32_t)cdiv(nin, group);
       uint32_t* out = nout == 1 ? s.W : dst;
+#if MSM_SUM_WARP
+      k_sum_groups_warp<C><<<(unsigned)cdiv((size_t)s.nset * nout * 32, 128), 128, 0, st>>>(src, nin, group, nout, s.nset, out);
+#else
       k_sum_groups<C><<<(unsigned)cdiv((size_t)s.nset * nout, 128), 128, 0, st>>>(src, nin, group, nout, s.nset, out);
+#endif
       launches++;
       nin = nout;
       std::swap(src, dst);
