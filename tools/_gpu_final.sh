@@ -1,7 +1,7 @@
 #!/bin/bash
 # Round-end evidence at HEAD (one B200): GPU tests, smoke, default bench, configs, launch list.
 cd "$(dirname "$0")/.."
-o=gpurun_out/final2; mkdir -p $o
+o=${OUT:-gpurun_out/final2}; mkdir -p $o
 timeout 900 python -m pytest tests -m gpu -x -q > $o/gpu_tests.log 2>&1
 timeout 300 python -c "import __graft_entry__ as g; g.smoke()" > $o/smoke.log 2>&1
 timeout 600 python bench.py > $o/bench_default.json 2> $o/bench_default.err
