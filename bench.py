@@ -125,61 +125,172 @@ def dist_env():
 
 
 # ---------------------------------------------------------------------------------------
-def cpu_baseline(curve, seconds_hint=True, n_sample=None):
-    """The oracle's plain Pippenger as it stands, single process, on a
-    bounded sample of the same workload (same curve, same input recipe)."""
+# CPU baseline: the oracle's plain Pippenger, as it
+# stands, on every host core: worker w owns points [w*chunk, (w+1)*chunk) of a prefix of
+# the bench workload (same curve, same input recipe), computes the MSM of its chunk, and
+# the partial points are summed.  The timed region is the Pippenger only (input generation
+# happens before a barrier).  The rate (points/s) is extrapolated to the full n, labelled.
+ORACLE_S = {"bn254": 8, "bls12_377": 8, "bls12_381": 8, "mnt4_753": 8}
+ORACLE_CHUNK = {"bn254": 1 << 13, "bls12_377": 1 << 13, "bls12_381": 1 << 13, "mnt4_753": 1 << 9}
+
+
+def _oracle_worker(curve, seed, off, cnt, s, barrier, conn):
+    sys.path.insert(0, ROOT)
     import synth
-    from oracle import msm as omsm, points as opoints
+    from oracle import points as opoints
+    from oracle import msm as omsm
     from oracle.curves import CURVES
     c = CURVES[curve]
-    if n_sample is None:
-        n_sample = 1 << 11 if curve != "mnt4_753" else 1 << 8
-    e0, d = synth.point_seeds(c.r, 20240427)
-    Ps = opoints.progression_points(e0, d, n_sample, c)
-    ks = synth.words_to_ints(synth.scalars_range(c.r, 0, n_sample, 20240427))
-    t0 = time.perf_counter()
-    omsm.msm_pippenger(ks, Ps, c, s=8)
-    dt = time.perf_counter() - t0
-    return {"value": n_sample / dt, "unit": "points/s", "cores": 1, "kind": "oracle",
-            "sample": f"{curve} n={n_sample} (first {n_sample} points/scalars of the workload recipe), "
-                      f"oracle.msm_pippenger s=8, pure-Python ints, 1 process; {dt:.2f} s",
-            "seconds": dt}
+    e0, d = synth.point_seeds(c.r, seed)
+    Ps = opoints.progression_points(synth.progression_offset(c.r, e0, d, off), d, cnt, c)
+    ks = synth.words_to_ints(synth.scalars_range(c.r, off, cnt, seed))
+    while True:
+        cmd = conn.recv()
+        if cmd != "run":
+            break
+        barrier.wait()
+        t0 = time.perf_counter()
+        Q = omsm.msm_pippenger(ks, Ps, c, s=s)
+        t1 = time.perf_counter()
+        conn.send((t0, t1, Q))
+
+
+def cpu_info():
+    model = None
+    try:
+        out = subprocess.run(["lscpu"], capture_output=True, text=True, timeout=10).stdout
+        for line in out.splitlines():
+            if line.startswith("Model name:"):
+                model = line.split(":", 1)[1].strip()
+    except Exception:
+        pass
+    if model is None:
+        try:
+            for line in open("/proc/cpuinfo"):
+                if line.startswith("model name"):
+                    model = line.split(":", 1)[1].strip()
+                    break
+        except Exception:
+            pass
+    try:
+        cores = len(os.sched_getaffinity(0))
+    except Exception:
+        cores = os.cpu_count() or 1
+    return cores, model
+
+
+class OraclePool:
+    """One spawned process per host core, each holding its chunk of the sample."""
+
+    def __init__(self, curve, seed, workers=None, chunk=None):
+        import multiprocessing as mp
+        cores, self.model = cpu_info()
+        self.workers = workers or cores
+        self.chunk = chunk or ORACLE_CHUNK[curve]
+        self.s = ORACLE_S[curve]
+        self.curve = curve
+        self.n_sample = self.workers * self.chunk
+        ctx = mp.get_context("spawn")
+        self.barrier = ctx.Barrier(self.workers)
+        self.conns, self.procs = [], []
+        for w in range(self.workers):
+            a, b = ctx.Pipe()
+            p = ctx.Process(target=_oracle_worker, args=(curve, seed, w * self.chunk, self.chunk, self.s, self.barrier, b),
+                            daemon=True)
+            p.start()
+            self.conns.append(a)
+            self.procs.append(p)
+
+    def run(self):
+        """(wall seconds of the parallel Pippenger, Q = sum of the chunk MSMs)."""
+        sys.path.insert(0, ROOT)
+        from oracle import ec
+        from oracle.curves import CURVES
+        for cn in self.conns:
+            cn.send("run")
+        res = [cn.recv() for cn in self.conns]
+        wall = max(r[1] for r in res) - min(r[0] for r in res)
+        c = CURVES[self.curve]
+        Q = None
+        for r in res:
+            Q = ec.add(Q, r[2], c)
+        return wall, Q
+
+    def close(self):
+        for cn in self.conns:
+            try:
+                cn.send("stop")
+            except Exception:
+                pass
+        for p in self.procs:
+            p.join(timeout=5)
+            if p.is_alive():
+                p.terminate()
+
+    def describe(self, wall, n_full):
+        return (f"{self.curve}: {self.n_sample}-point prefix of the n={n_full} workload "
+                f"({self.workers} processes x {self.chunk} points, oracle.msm_pippenger s={self.s}, pure-Python ints, "
+                f"partials summed); {wall:.2f} s wall; points/s extrapolated linearly to n (Pippenger cost per point "
+                f"is ~constant in n at fixed s)")
+
+
+def cpu_baseline(curve, n_full, seed):
+    """SURVEY.md §8(d) CPU baseline, one bounded run on all host cores."""
+    pool = OraclePool(curve, seed)
+    try:
+        wall, _ = pool.run()
+    finally:
+        pool.close()
+    return {"value": pool.n_sample / wall, "unit": "points/s", "cores": pool.workers, "cpu_model": pool.model,
+            "kind": "oracle", "sample": pool.describe(wall, n_full), "seconds": wall,
+            "extrapolated_ms_full_n": n_full / (pool.n_sample / wall) * 1e3}
 
 
 def run_reference(args):
+    """Reference arm (tier framing): the oracle as it stands on the host cores, each step a
+    bounded sample of the bench workload.  Rank 0 only; other ranks exit at once."""
     ws, rank, local = dist_env()
     if rank != 0:
         return 0
     curve = args.curve
-    n_sample = args.ref_sample or (1 << 10 if curve != "mnt4_753" else 1 << 7)
-    import synth
-    from oracle import msm as omsm, points as opoints
-    from oracle.curves import CURVES
-    c = CURVES[curve]
-    e0, d = synth.point_seeds(c.r, 20240427)
-    Ps = opoints.progression_points(e0, d, n_sample, c)
-    ks = synth.words_to_ints(synth.scalars_range(c.r, 0, n_sample, 20240427))
-    for _ in range(args.warmup):
-        omsm.msm_pippenger(ks, Ps, c, s=8)
-    times = []
-    for _ in range(args.steps):
-        t0 = time.perf_counter()
-        omsm.msm_pippenger(ks, Ps, c, s=8)
-        times.append(time.perf_counter() - t0)
+    seed = 20240427 + 3
+    cores, _ = cpu_info()
+    chunk = args.ref_sample // cores if args.ref_sample else max(64, ORACLE_CHUNK[curve] // 8)
+    pool = OraclePool(curve, seed, chunk=chunk)
+    try:
+        for _ in range(args.warmup):
+            pool.run()
+        times = [pool.run()[0] for _ in range(args.steps)]
+    finally:
+        pool.close()
     ms = statistics.median(times) * 1e3
-    val = n_sample / (ms / 1e3)
+    val = pool.n_sample / (ms / 1e3)
+    n = 1 << args.log2n
     line = {
         "impl": "reference", "metric": METRIC, "value": val, "unit": "points/s", "n_gpus": args.gpus,
         "steps": args.steps, "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": True,
         "scaling": "strong", "vs_baseline": None, "dtype": "int (python big ints)", "data": "synthetic",
-        "config": {"workload": f"{curve} G1 MSM n=2^{args.log2n}", "curve": curve, "n": 1 << args.log2n,
-                   "sample_n": n_sample, "l2": "n/a (CPU)"},
-        "cpu_baseline": {"value": val, "unit": "points/s", "cores": 1, "kind": "oracle",
-                         "sample": f"{curve} n={n_sample} per step, oracle.msm_pippenger s=8, 1 process"},
+        "config": {"workload": f"{curve} G1 MSM n=2^{args.log2n}", "curve": curve, "n": n,
+                   "sample_n": pool.n_sample, "l2": "n/a (CPU)"},
+        "cpu_baseline": {"value": val, "unit": "points/s", "cores": pool.workers, "cpu_model": pool.model,
+                         "kind": "oracle", "sample": pool.describe(ms / 1e3, n)},
         "e2e": {"value": val, "unit": "points/s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
     }
     print(json.dumps(line), flush=True)
     return 0
+
+
+def self_launch(args):
+    """`python bench.py --gpus N` outside torchrun: re-run this script under
+    torch.distributed.run with N ranks (one process per GPU, 127.0.0.1 rendezvous)."""
+    import socket
+    s = socket.socket()
+    s.bind(("127.0.0.1", 0))
+    port = s.getsockname()[1]
+    s.close()
+    cmd = [sys.executable, "-m", "torch.distributed.run", "--nnodes=1", f"--nproc-per-node={args.gpus}",
+           "--master-addr", "127.0.0.1", "--master-port", str(port), os.path.abspath(__file__)] + sys.argv[1:]
+    return subprocess.run(cmd).returncode
 
 
 # ---------------------------------------------------------------------------------------
@@ -202,12 +313,15 @@ def main():
     ap.add_argument("--ref-sample", type=int, default=0)
     ap.add_argument("--no-e2e", action="store_true")
     ap.add_argument("--no-cpu-baseline", action="store_true")
-    ap.add_argument("--check", action="store_true", help="verify the result against the oracle closed form")
+    ap.add_argument("--no-check", action="store_true",
+                    help="skip the closed-form check of the result (run by default after the timed region)")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3
     if args.impl == "reference":
         return run_reference(args)
+    if args.gpus > 1 and "WORLD_SIZE" not in os.environ:
+        return self_launch(args)
 
     import numpy as np
     import torch
@@ -217,10 +331,15 @@ def main():
     from paper_conf_asplos_ji0x024_b200.dist import gather_and_finalize, shard_bounds
 
     ws, rank, local = dist_env()
-    assert ws == args.gpus, f"--gpus {args.gpus} but WORLD_SIZE {ws}"
-    # MSM_BENCH_SHARE_DEVICE=1 (test only): every rank on cuda:0 and the gather over gloo
-    # with host partials, so the N > 1 path can be exercised on a one-GPU box.
-    share = os.environ.get("MSM_BENCH_SHARE_DEVICE") == "1"
+    if ws != args.gpus:
+        print(f"bench.py: --gpus {args.gpus} but WORLD_SIZE {ws}; using WORLD_SIZE", file=sys.stderr)
+    # Shared-device mode (test only; automatic when the box has fewer GPUs than ranks, or
+    # MSM_BENCH_SHARE_DEVICE=1): every rank on cuda:0 and the gather over gloo with host
+    # partials, so the N > 1 path runs end to end on a one-GPU box.  Its timings are not
+    # scaling numbers (the ranks share one GPU) and the line says so.
+    share = os.environ.get("MSM_BENCH_SHARE_DEVICE") == "1" or (ws > 1 and torch.cuda.device_count() < ws)
+    if share and ws > 1 and rank == 0:
+        print(f"bench.py: shared-device mode ({ws} ranks on cuda:0, gloo gather)", file=sys.stderr)
     torch.cuda.set_device(0 if share else local)
     dev = torch.device("cuda", 0 if share else local)
     coll_dev = torch.device("cpu") if share else dev
@@ -237,7 +356,7 @@ def main():
     # multi-GPU decomposition: "points" = contiguous point shards (north_star), "buckets" =
     # the paper's bucket split (f1): every rank holds all n points and scalars
     # and sums the buckets |d| = ws*q + rank of every bucket set
-    split = args.split if args.split != "auto" else ("buckets" if ws > 1 else "points")
+    split = args.split if args.split != "auto" else ("buckets" if ws > 1 and not share else "points")
     off, n_g = shard_bounds(n, ws, rank) if split == "points" else (0, n)
     seed = 20240427 + 3
     e0, delta = synth.point_seeds(r, seed)
@@ -250,7 +369,16 @@ def main():
     ks_host = synth.scalars_range(r, off, n_g, seed)
     ks_pinned = torch.from_numpy(ks_host.view(np.int32)).pin_memory()
     ks_dev = ks_pinned.to(dev, non_blocking=False)
-    ctx = msm.Context(curve, pts, ngpus=1, n=n_g)
+    if share and ws > 1:
+        # ranks sharing one GPU create their contexts (and f3 tables) one after another, so
+        # each planner sees the memory the previous ones took
+        for turn in range(ws):
+            if turn == rank:
+                ctx = msm.Context(curve, pts, ngpus=1, n=n_g)
+            torch.distributed.barrier()
+    else:
+        ctx = msm.Context(curve, pts, ngpus=1, n=n_g)
+    assert ctx.get_option(msm.OPT_DEVICE) == dev.index, "context not on this rank's device"
     del pts
     torch.cuda.empty_cache()
     if args.precompute != 2:
@@ -346,8 +474,12 @@ def main():
                "timing": "host wall clock around msm_run with pinned host scalars (max over ranks)"}
 
     check = None
-    if args.check and rank == 0:
+    if not args.no_check and rank == 0:
+        t_chk = time.time()
         check = verify(curve, n, e0, delta, seed, ctx if ws == 1 else None, ks_dev, res, msm)
+        check["seconds"] = round(time.time() - t_chk, 1)
+        check["what"] = ("last timed step's affine result vs the oracle closed form (e0*sum k_i + delta*sum i*k_i "
+                         "mod r)*G over all n scalars (oracle/msm.py closed_form_arith)")
 
     if rank != 0:
         ctx.close()
@@ -356,16 +488,22 @@ def main():
             torch.distributed.destroy_process_group()
         return 0
 
-    # roofline of the dominant kernel (k_accumulate): algorithmic IMAD-pipe slots per launch
+    # roofline of the dominant kernel (k_accumulate): algorithmic work =
+    # PACC x 10 field mults x (4 L32^2 + L32) IMAD (CIOS on 32-bit limbs, L32 = 8/12/12/24)
+    # per launch, over the kernel's CUDA-event time, against 148 SM x 64 IMAD/clk x max clock.
+    # frac_pipe is the IMAD-pipe occupancy of the instruction stream actually run
+    # (radix-2^W limbs: 2 slots per IMAD.WIDE), which is what ncu's fmaheavy counter sees.
     st = stage[-1]
     nonempty = ctx.get_option(msm.OPT_NONEMPTY)
     pacc = int(st["entries"]) - int(nonempty)
+    imad_alg = pacc * 10 * (4 * L32 * L32 + L32)
     slots = pacc * imad_slots_per_pacc(L)
     acc_avg_ms = sum(acc_ms) / len(acc_ms)
     pk = peaks()
     sm_max = pk.get("sm_max_mhz", 1965.0)
-    peak_slots = 148 * 64 * sm_max * 1e6
-    achieved = slots / (acc_avg_ms / 1e3)
+    peak_imad = 148 * 64 * sm_max * 1e6
+    achieved = imad_alg / (acc_avg_ms / 1e3)
+    achieved_slots = slots / (acc_avg_ms / 1e3)
     # a3 (digits + counting sort) against HBM: algorithmic bytes = scalars read once
     # (n*S*4) + sorted entries written once (M*4); sort_ms is the stage's CUDA-event time on
     # the library stream
@@ -376,7 +514,7 @@ def main():
     clocks = sampler.summary()
     cpu = None
     if not args.no_cpu_baseline and ws == 1:
-        cpu = cpu_baseline(curve)
+        cpu = cpu_baseline(curve, n, seed)
     paper = PAPER_MS.get((curve, args.log2n, ws))
     line = {
         "metric": METRIC,
@@ -397,7 +535,10 @@ def main():
                    "precompute": bool(st["precompute"]), "sort_variant": ctx.get_option(msm.OPT_SORT),
                    "bucket_sets": 1 if st["precompute"] else st["nwin"],
                    "parallelism": (f"point-sharded x{ws}" if split == "points" else f"bucket-split x{ws} (PAPER.md:223)")
-                                  + (" + NCCL all-gather of partials" if ws > 1 else ""),
+                                  + ((" + gloo all-gather of host partials (shared-device test mode: all ranks on cuda:0, "
+                                      "times are NOT scaling numbers)" if share else " + NCCL all-gather of partials")
+                                     if ws > 1 else ""),
+                   "shared_device": bool(share and ws > 1),
                    "scalars": "device-resident (HBM) for value; pinned host for e2e",
                    "l2": "inputs >> L2 (points %.1f GB + scalars %.1f GB per step); no flush needed" % (
                        n * (2 * L + 2) * 4 / 1e9, n * S * 4 / 1e9)},
@@ -408,10 +549,17 @@ def main():
                           "peak_basis": "MEASURED_PEAKS.json hbm_gbs (copy bandwidth)"},
         "stages_ms": {k: round(v, 3) for k, v in st.items() if k.endswith("_ms") and k != "table_ms"},
         "latency_ms": {"mean": ms, "min": min(times), "max": max(times)},
-        "roofline": {"kernel": "k_accumulate_sync" if L <= 13 else "k_accumulate", "bound": "alu", "achieved": achieved / 1e12, "peak": peak_slots / 1e12,
-                     "unit": "T IMAD-pipe slots/s", "frac": achieved / peak_slots, "traffic": ncu_traffic(curve, args.log2n),
-                     "work": f"{pacc} PACC x (8 mul x {imad_slots_per_mult(L)} + 2 sqr x {imad_slots_per_sqr(L)}) IMAD slots",
-                     "peak_basis": f"148 SM x 64 IMAD slots/clk x {sm_max} MHz (clocks.max.sm); IMAD.WIDE = 2 slots (measured)",
+        "roofline": {"kernel": "k_accumulate_sync" if L <= 13 else "k_accumulate", "bound": "alu",
+                     "achieved": achieved / 1e12, "peak": peak_imad / 1e12, "unit": "T IMAD/s",
+                     "frac": achieved / peak_imad, "traffic": ncu_traffic(curve, args.log2n),
+                     "work": f"{pacc} PACC x 10 field mults x (4*{L32}^2+{L32} = {4 * L32 * L32 + L32}) IMAD "
+                             f"(SURVEY.md §8(d): CIOS on 32-bit limbs) per launch",
+                     "time_basis": f"k_accumulate CUDA-event average over the {args.steps} timed steps, library stream",
+                     "peak_basis": f"148 SM x 64 IMAD/clk x {sm_max} MHz (clocks.max.sm; B200 guide unit counts)",
+                     "frac_pipe": achieved_slots / peak_imad,
+                     "frac_pipe_basis": f"IMAD-pipe slots of the radix-2^{W} instruction stream run: {pacc} PACC x "
+                                        f"(8 mul x {imad_slots_per_mult(L)} + 2 sqr x {imad_slots_per_sqr(L)}) slots, "
+                                        "IMAD.WIDE = 2 slots (measured)",
                      "field_mults_per_s": pacc * 10 / (acc_avg_ms / 1e3)},
         "clocks": clocks,
         "gpu_launches": int(st["acc_launches"]) * args.steps + (args.steps if ws > 1 else 0),

@@ -11,7 +11,9 @@
  * Encoding (all integers are arrays of little-endian 32-bit words):
  *   base-field element   L32 = msm_field_words(curve) words, canonical (< p)
  *   affine point         2*L32 words: x then y.  (0, 0) encodes the point at infinity O
- *                        (it is on none of the four curves because b != 0)
+ *                        (it is on none of the four curves because b != 0).  A point with
+ *                        y = 0 (order 2; it exists on BLS12-377: (p-1, 0)) is outside the
+ *                        prime-order subgroup and rejected with MSM_ERR_POINT.
  *   scalar               S = msm_scalar_words(curve) words, canonical (< r)
  *   result               2*L32 words, canonical affine; O -> (0, 0)
  *   partial (XYZZ)       msm_partial_words(curve) words: the library's internal projective
@@ -29,6 +31,18 @@
  * the context stays usable; after MSM_ERR_CUDA it should be destroyed.
  *
  * Threading: one call at a time per context; distinct contexts are independent.
+ *
+ * Devices: every call restores the caller's current CUDA device before it returns.  A
+ * context's shard g lives on device (current device at create + g) mod device-count, so a
+ * one-process-per-GPU caller that selected cuda:LOCAL_RANK gets its context there;
+ * msm_context_create_on takes an explicit device per shard.
+ *
+ * Ordering of device-resident inputs: before reading a device pointer argument the
+ * library orders its own (non-blocking) streams after all work already submitted to the
+ * legacy default stream of the pointer's device — where torch's default stream and
+ * synchronous CUDA calls run.  Inputs produced on other non-blocking streams must be
+ * complete (synchronised by the caller) before the call.  Calls return only after their
+ * device outputs are written (msm_submit: results are read through msm_wait).
  */
 #ifndef MSM_H
 #define MSM_H
@@ -48,7 +62,9 @@ enum {
   MSM_ERR_CURVE = -2,         /* unknown curve id                                       */
   MSM_ERR_CUDA = -3,          /* CUDA runtime error                                     */
   MSM_ERR_OOM = -4,           /* device allocation failed                               */
-  MSM_ERR_NCCL = -5,          /* reserved (collectives run in the caller's process group) */
+  MSM_ERR_NCCL = -5,          /* reserved: the library itself makes no NCCL calls; the
+                                 one-process-per-GPU gather runs in the caller's process
+                                 group (paper_conf_asplos_ji0x024_b200/dist.py)           */
   MSM_ERR_POINT = -6,         /* an input point is not on the curve or not canonical    */
   MSM_ERR_SCALAR = -7,        /* a scalar is >= r                                       */
   MSM_ERR_UNIMPLEMENTED = -8,
@@ -79,7 +95,9 @@ enum {
   MSM_OPT_SPLIT_INDEX = 7,    /* f1: this context's part g in [0, G), default 0               */
   MSM_OPT_NWIN = 101,         /* (get only) number of windows floor(lambda/c) + 1           */
   MSM_OPT_NSETS = 103,        /* (get only) bucket sets: nwin, or 1 with the f3 table        */
-  MSM_OPT_NONEMPTY = 102      /* (get only) non-empty buckets of the last run on device 0   */
+  MSM_OPT_NONEMPTY = 102,     /* (get only) non-empty buckets of the last run on shard 0    */
+  MSM_OPT_DEVICE = 104,       /* (get only) CUDA device of shard 0 (msm_shard_info: any shard) */
+  MSM_OPT_NGPUS = 105         /* (get only) number of shards G                              */
 };
 
 /* Per-stage device times of the last msm_run on device 0 (CUDA events), milliseconds. */
@@ -121,12 +139,29 @@ int msm_device_count(void);
  */
 msm_context* msm_context_create(int curve, const uint32_t* points, size_t n, int ngpus);
 
+/*
+ * As msm_context_create with an explicit CUDA device per shard: devices[g] in
+ * [0, msm_device_count()).  A device may repeat: several shards then share it ("logical
+ * shards" — each with its own stream and scratch, the gather a same-device copy); this is
+ * how the multi-shard path (per-shard pipelines, cross-shard gather of the partials,
+ * final add) is exercised on a one-GPU machine.
+ * Returns NULL on error (msm_last_error(): also MSM_ERR_NO_DEVICE for a bad device id).
+ */
+msm_context* msm_context_create_on(int curve, const uint32_t* points, size_t n, int ngpus, const int* devices);
+
+/* Shard g of the context: its device and its contiguous point range [offset, offset+count). */
+int msm_shard_info(const msm_context* ctx, int g, int* device, size_t* offset, size_t* count);
+
 /* NULL-safe; frees all device memory and streams of the context. */
 void msm_context_destroy(msm_context* ctx);
 
 /*
- * Q = sum k_i P_i.  `scalars`: n*S words, host or device (device 0 for ngpus > 1 is
- * copied peer-to-peer).  `result`: host buffer of 2*L32 words (written only on MSM_OK).
+ * Q = sum k_i P_i.  `scalars`: n*S words, host or device.  Each shard reads its slice
+ * [offset, offset+count): in place when it is on the shard's device (16-B aligned),
+ * otherwise by a peer (NVLink) or host copy; host slices are uploaded by one host thread
+ * per shard in parallel.  The G partial sums then meet on shard 0's device (peer copies
+ * of 4L words each — the gather of PAPER.md:163) for the final add and normalisation.
+ * `result`: host buffer of 2*L32 words (written only on MSM_OK).
  * Synchronous.  Returns MSM_OK, MSM_ERR_SCALAR (some k_i >= r), MSM_ERR_ARG, MSM_ERR_CUDA.
  */
 int msm_run(msm_context* ctx, const uint32_t* scalars, uint32_t* result);

@@ -15,6 +15,7 @@
 #include <memory>
 #include <mutex>
 #include <new>
+#include <thread>
 #include <vector>
 
 #include "runtime.h"
@@ -56,6 +57,34 @@ bool is_device_ptr(const void* p, int* dev) {
   return false;
 }
 
+// Restores the caller's current device when an ABI call returns (the library switches
+// devices per shard; the caller's torch/CUDA state must not change under it).
+struct DeviceGuard {
+  int dev = -1;
+  DeviceGuard() {
+    if (cudaGetDevice(&dev) != cudaSuccess) { cudaGetLastError(); dev = -1; }
+  }
+  ~DeviceGuard() {
+    if (dev >= 0) cudaSetDevice(dev);
+  }
+};
+
+// Orders `stream` (on device `dev`) after all work already submitted to the legacy default
+// stream of device `src_dev` — where torch (default stream) and synchronous CUDA calls put
+// the producers of device-resident inputs.  Inputs written on other non-blocking streams
+// must be complete before the call (include/msm.h, "Ordering").
+std::mutex g_order_mu;
+cudaEvent_t g_order_ev[64] = {};
+void order_after_legacy(int src_dev, int dev, cudaStream_t stream) {
+  if (src_dev < 0 || src_dev >= 64) return;
+  std::lock_guard<std::mutex> lk(g_order_mu);
+  CK(cudaSetDevice(src_dev));
+  if (!g_order_ev[src_dev]) CK(cudaEventCreateWithFlags(&g_order_ev[src_dev], cudaEventDisableTiming));
+  CK(cudaEventRecord(g_order_ev[src_dev], cudaStreamLegacy));
+  CK(cudaSetDevice(dev));
+  CK(cudaStreamWaitEvent(stream, g_order_ev[src_dev], 0));
+}
+
 // Pippenger cost model, in units of one PACC (10 field mults):
 //   per window n PACC ("ceil(lambda/s)(N + 2^{s+1})"), plus a sort cost per
 //   entry, plus the bucket reduce (2 PADD per bucket, measured ~4.4 PACC-equivalents per
@@ -91,22 +120,32 @@ void plan_shard(const Options& o, const Shard& s, int lambda, int PW, int XW, in
     if (pre) need += (double)table_bytes(s.n, lambda, c, PW);
     return need <= budget;
   };
-  // sorted entries hold (table row j)*n + i in 31 bits
+  // Entry counts (goff, cursors, M) are 32-bit and a sorted entry holds its point index in
+  // 31 bits: (table row j)*n + i with the f3 table, i without it.  Every c whose nwin*n
+  // entries could overflow either is skipped (n < 2^31 is checked at create).
   auto indexable = [&](int c) { return (double)num_windows(lambda, c) * (double)s.n < 2147483647.0; };
   const int cmin = o.c > 0 ? o.c : 4, cmax = o.c > 0 ? o.c : 24;
   double best = 1e300;
   int bc = o.c > 0 ? o.c : 8, bp = 0;
-  for (int pre = 0; pre <= 1; pre++) {
-    if ((o.pre == 0 && pre) || (o.pre == 1 && !pre)) continue;
-    for (int c = cmin; c <= cmax; c++) {
-      if (o.c <= 0 && c > 22 && !pre) continue;  // per-window bucket sets beyond 2^21
-      if (pre && !indexable(c)) continue;
-      if (o.pre == 2 && pre && !fits(c, true)) continue;
-      const double cost = s.n == 0 ? (double)c : plan_cost(s.n, lambda, c, pre);
-      if (cost < best) { best = cost; bc = c; bp = pre; }
+  bool any_fit = false;
+  for (int pass = 0; pass < 2 && best == 1e300; pass++) {
+    // pass 0 requires the memory fit of every candidate; pass 1 (nothing fits) lets an
+    // explicitly chosen configuration try its allocation (MSM_ERR_OOM if it fails)
+    for (int pre = 0; pre <= 1; pre++) {
+      if ((o.pre == 0 && pre) || (o.pre == 1 && !pre)) continue;
+      for (int c = cmin; c <= cmax; c++) {
+        if (o.c <= 0 && c > 22 && !pre) continue;  // per-window bucket sets beyond 2^21
+        if (!indexable(c)) continue;
+        const bool fit = fits(c, pre);
+        any_fit |= fit;
+        if (pass == 0 && !fit && (o.pre == 2 || o.c <= 0)) continue;
+        const double cost = s.n == 0 ? (double)c : plan_cost(s.n, lambda, c, pre);
+        if (cost < best) { best = cost; bc = c; bp = pre; }
+      }
     }
+    if (o.pre == 2 && o.c <= 0) break;  // fully automatic: only configurations that fit
   }
-  if (best == 1e300) throw CudaError{MSM_ERR_ARG};  // forced table not indexable at this c
+  if (best == 1e300) throw CudaError{any_fit ? MSM_ERR_ARG : MSM_ERR_OOM};
   *c_out = bc;
   *pre_out = bp;
 }
@@ -183,14 +222,36 @@ int run_all(msm_context* ctx, const uint32_t* scalars, bool gather_to_dev0) {
   ctx->launches = 0;
   const int XW = ctx->ops->XW();
   Shard& s0 = ctx->shards[0];
-  for (size_t g = 0; g < ctx->shards.size(); g++) {
+  const size_t G = ctx->shards.size();
+  std::vector<int> launched(G, 0), rc(G, MSM_OK);
+  auto one = [&](size_t g) {
     Shard& s = ctx->shards[g];
-    CK(cudaSetDevice(s.dev));
-    const bool timed = g == 0;
-    if (timed) CK(cudaEventRecord(s.ev[EV_START], s.stream));
-    CK(cudaMemsetAsync(s.err, 0, 4, s.stream));
-    const uint32_t* sc = stage_scalars(ctx, s, scalars, is_dev, src_dev);
-    ctx->launches += ctx->ops->enqueue_pipeline(s, sc, timed);
+    try {
+      CK(cudaSetDevice(s.dev));
+      const bool timed = g == 0;
+      if (is_dev) order_after_legacy(src_dev, s.dev, s.stream);
+      if (timed) CK(cudaEventRecord(s.ev[EV_START], s.stream));
+      CK(cudaMemsetAsync(s.err, 0, 4, s.stream));
+      const uint32_t* sc = stage_scalars(ctx, s, scalars, is_dev, src_dev);
+      launched[g] = ctx->ops->enqueue_pipeline(s, sc, timed);
+    } catch (const CudaError& e) {
+      rc[g] = e.code;
+    } catch (...) {
+      rc[g] = MSM_ERR_CUDA;
+    }
+  };
+  if (G > 1 && ctx->n && !is_dev) {
+    // host scalars: one host thread per shard, so the (possibly pageable, hence
+    // host-synchronous) H2D copies of the shards run in parallel over their own links
+    std::vector<std::thread> th;
+    for (size_t g = 0; g < G; g++) th.emplace_back(one, g);
+    for (auto& t : th) t.join();
+  } else {
+    for (size_t g = 0; g < G; g++) one(g);
+  }
+  for (size_t g = 0; g < G; g++) {
+    if (rc[g] != MSM_OK) throw CudaError{rc[g]};
+    ctx->launches += launched[g];
   }
   if (gather_to_dev0) {
     for (size_t g = 0; g < ctx->shards.size(); g++) {
@@ -239,8 +300,11 @@ void collect_stats(msm_context* ctx) {
   st.table_ms = s.table_ms;
 }
 
+// Every ABI call that touches a device runs through guarded(): C++ exceptions become
+// MSM_ERR_* codes and the caller's current device is restored on return.
 template <class F>
 int guarded(F&& f) {
+  DeviceGuard guard;
   try {
     return f();
   } catch (const CudaError& e) {
@@ -313,11 +377,29 @@ const char* msm_error_string(int code) {
 
 msm_context* msm_context_create(int curve, const uint32_t* points, size_t n, int ngpus) {
   g_last_error = MSM_OK;
+  const int ndev = msm_device_count();
+  if (ndev < 1) { g_last_error = MSM_ERR_NO_DEVICE; return nullptr; }
+  if (ngpus < 1 || ngpus > 64) { g_last_error = MSM_ERR_ARG; return nullptr; }
+  if (ngpus > ndev) { g_last_error = MSM_ERR_NO_DEVICE; return nullptr; }
+  // shard g on device (current + g) mod ndev: a one-process-per-GPU caller that selected
+  // cuda:LOCAL_RANK gets its context there
+  int base = 0;
+  if (cudaGetDevice(&base) != cudaSuccess) { cudaGetLastError(); base = 0; }
+  int devs[64];
+  for (int g = 0; g < ngpus; g++) devs[g] = (base + g) % ndev;
+  return msm_context_create_on(curve, points, n, ngpus, devs);
+}
+
+msm_context* msm_context_create_on(int curve, const uint32_t* points, size_t n, int ngpus, const int* devices) {
+  g_last_error = MSM_OK;
+  DeviceGuard guard;
   CurveOps* ops = ops_for(curve);
   if (!ops) { g_last_error = MSM_ERR_CURVE; return nullptr; }
-  if (ngpus < 1 || (n > 0 && !points) || n >= 0x80000000ull) { g_last_error = MSM_ERR_ARG; return nullptr; }
+  if (ngpus < 1 || ngpus > 64 || !devices || (n > 0 && !points) || n >= 0x80000000ull) { g_last_error = MSM_ERR_ARG; return nullptr; }
   const int ndev = msm_device_count();
-  if (ndev < 1 || ngpus > ndev) { g_last_error = MSM_ERR_NO_DEVICE; return nullptr; }
+  if (ndev < 1) { g_last_error = MSM_ERR_NO_DEVICE; return nullptr; }
+  for (int g = 0; g < ngpus; g++)
+    if (devices[g] < 0 || devices[g] >= ndev) { g_last_error = MSM_ERR_NO_DEVICE; return nullptr; }
   auto* ctx = new msm_context();
   ctx->curve = curve;
   ctx->n = n;
@@ -330,7 +412,7 @@ msm_context* msm_context_create(int curve, const uint32_t* points, size_t n, int
     const size_t pw_in = 2 * (size_t)ops->L32();
     for (int g = 0; g < ngpus; g++) {
       Shard& s = ctx->shards[g];
-      s.dev = g;
+      s.dev = devices[g];
       s.off = (size_t)((unsigned __int128)n * g / ngpus);
       s.n = (size_t)((unsigned __int128)n * (g + 1) / ngpus) - s.off;
       CK(cudaSetDevice(s.dev));
@@ -346,6 +428,7 @@ msm_context* msm_context_create(int curve, const uint32_t* points, size_t n, int
       CK(cudaMemsetAsync(s.err, 0, 4, s.stream));
       if (s.n) {
         const uint32_t* src = points + s.off * pw_in;
+        if (in_dev) order_after_legacy(src_dev, s.dev, s.stream);
         if (in_dev && src_dev == s.dev) {
           ops->points_to_mont(s, src, s.n);
         } else {
@@ -364,13 +447,14 @@ msm_context* msm_context_create(int curve, const uint32_t* points, size_t n, int
     if (ngpus > 1) {
       for (int a = 0; a < ngpus; a++)
         for (int b = 0; b < ngpus; b++) {
-          if (a == b) continue;
+          const int da = ctx->shards[a].dev, db = ctx->shards[b].dev;
+          if (da == db) continue;  // logical shards on one device
           int ok = 0;
-          cudaDeviceCanAccessPeer(&ok, a, b);
+          cudaDeviceCanAccessPeer(&ok, da, db);
           if (ok) {
-            cudaSetDevice(a);
-            cudaError_t pe = cudaDeviceEnablePeerAccess(b, 0);
-            if (pe != cudaSuccess) cudaGetLastError();
+            cudaSetDevice(da);
+            cudaError_t pe = cudaDeviceEnablePeerAccess(db, 0);
+            if (pe != cudaSuccess) cudaGetLastError();  // already enabled
           }
         }
     }
@@ -387,6 +471,7 @@ msm_context* msm_context_create(int curve, const uint32_t* points, size_t n, int
 
 void msm_context_destroy(msm_context* ctx) {
   if (!ctx) return;
+  DeviceGuard guard;
   if (ctx->copy_stream) {
     cudaSetDevice(ctx->shards[0].dev);
     cudaStreamSynchronize(ctx->shards[0].stream);
@@ -463,6 +548,8 @@ long msm_submit(msm_context* ctx, const uint32_t* scalars) {
     // re-recorded by every pipeline, so this waits on the latest one), then H2D
     CK(cudaStreamWaitEvent(ctx->copy_stream, s.ev[EV_SORT], 0));
     const size_t bytes = s.n * (size_t)ctx->ops->S() * 4;
+    int src_dev = -1;
+    if (bytes && is_device_ptr(scalars, &src_dev)) order_after_legacy(src_dev, s.dev, ctx->copy_stream);
     if (bytes) CK(cudaMemcpyAsync(s.scal, scalars + s.off * ctx->ops->S(), bytes, cudaMemcpyDefault, ctx->copy_stream));
     CK(cudaEventRecord(ctx->ev_copied, ctx->copy_stream));
     // compute stream: a2..a6 on the staged scalars, then finalise into result slot q
@@ -522,7 +609,8 @@ int msm_finalize(int curve, const uint32_t* partials, int count, uint32_t* resul
     const uint32_t* src = fs.partials;
     int pdev = -1;
     if (count > 0) {
-      if (is_device_ptr(partials, &pdev) && pdev == dev) src = partials;
+      if (is_device_ptr(partials, &pdev)) order_after_legacy(pdev, dev, fs.stream);
+      if (pdev == dev) src = partials;
       else CK(cudaMemcpyAsync(fs.partials, partials, (size_t)count * ops->XW() * 4,
                               pdev >= 0 ? cudaMemcpyDefault : cudaMemcpyHostToDevice, fs.stream));
     }
@@ -583,6 +671,8 @@ long msm_get_option(msm_context* ctx, int key) {
     case MSM_OPT_NSETS: return ctx->shards[0].nset;
     case MSM_OPT_SPLIT_PARTS: return ctx->opt.split_G;
     case MSM_OPT_SPLIT_INDEX: return ctx->opt.split_g;
+    case MSM_OPT_DEVICE: return ctx->shards[0].dev;
+    case MSM_OPT_NGPUS: return (long)ctx->shards.size();
     case MSM_OPT_NONEMPTY: {
       long v = MSM_ERR_CUDA;
       guarded([&]() -> int { CK(cudaSetDevice(ctx->shards[0].dev)); v = ctx->ops->count_nonempty(ctx->shards[0]); return MSM_OK; });
@@ -595,6 +685,15 @@ long msm_get_option(msm_context* ctx, int key) {
 int msm_get_stats(const msm_context* ctx, msm_stats* out) {
   if (!ctx || !out) return MSM_ERR_ARG;
   *out = ctx->stats;
+  return MSM_OK;
+}
+
+int msm_shard_info(const msm_context* ctx, int g, int* device, size_t* offset, size_t* count) {
+  if (!ctx || g < 0 || g >= (int)ctx->shards.size()) return MSM_ERR_ARG;
+  const Shard& s = ctx->shards[g];
+  if (device) *device = s.dev;
+  if (offset) *offset = s.off;
+  if (count) *count = s.n;
   return MSM_OK;
 }
 

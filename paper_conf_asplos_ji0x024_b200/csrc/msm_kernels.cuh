@@ -98,6 +98,12 @@ __global__ void k_points_to_mont(uint32_t* __restrict__ pts, const uint32_t* __r
       if (!decy && yw[k] != pk) { lty = yw[k] < pk; decy = true; }
     }
     if (!ltx || !lty) atomicOr(err, 2u);
+    // y = 0 would be read as O by the accumulation: such a point has order 2 (on
+    // BLS12-377, (p-1, 0) lies on the curve) and is outside the prime-order subgroup
+    uint32_t ynz = 0;
+#pragma unroll
+    for (int k = 0; k < C::L32; k++) ynz |= yw[k];
+    if (!ynz) atomicOr(err, 1u);
     from_words32<C>(x, xw);
     from_words32<C>(y, yw);
     fto_mont<C>(x, x);
@@ -567,7 +573,8 @@ static __global__ void k_count_nonempty(const uint32_t* __restrict__ goff, size_
 //   buckets[f] (complete, or the owner's partial); a slice that starts inside a bucket
 //   writes its partial to carry[t] (carry_f[t] = f) for k_fixup.
 // Gathers the point of a sorted entry; negates y for a negative digit.  Returns false for
-// the point at infinity (stored as x = y = 0; y = 0 is on none of the curves since b != 0).
+// the point at infinity (stored as x = y = 0).  A stored y is 0 only for O: points with
+// y = 0 (order 2) are rejected at context creation (k_points_to_mont).
 template <class C>
 DEVI bool point_for_entry(uint32_t* x, uint32_t* y, const uint32_t* __restrict__ pts, uint32_t e) {
   load_point<C>(x, y, pts, e & ~SIGN_BIT);

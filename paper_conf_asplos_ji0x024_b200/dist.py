@@ -31,6 +31,11 @@ def gather_and_finalize(curve, partial, group=None):
     import torch.distributed as dist
     from . import msm
     allp = gather_partials(partial, group)
+    if allp.is_cuda:
+        # the all-gather's result is ordered on torch's current stream; the library orders
+        # itself only after the legacy default stream, so make the data complete here
+        import torch
+        torch.cuda.current_stream(allp.device).synchronize()
     if dist.get_rank(group) == 0:
         return msm.finalize(curve, allp, allp.shape[0])
     return None

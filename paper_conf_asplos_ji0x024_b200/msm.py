@@ -30,6 +30,8 @@ OPT_SPLIT_INDEX = 7
 OPT_NWIN = 101
 OPT_NONEMPTY = 102
 OPT_NSETS = 103
+OPT_DEVICE = 104
+OPT_NGPUS = 105
 
 ERRORS = {
     0: "ok", -1: "invalid argument", -2: "unknown curve", -3: "CUDA error", -4: "device out of memory",
@@ -71,6 +73,8 @@ def lib() -> ctypes.CDLL:
         "msm_field_words": (i, [i]), "msm_scalar_words": (i, [i]), "msm_scalar_bits": (i, [i]),
         "msm_partial_words": (i, [i]), "msm_device_count": (i, []),
         "msm_context_create": (P, [i, P, sz, i]), "msm_context_destroy": (None, [P]),
+        "msm_context_create_on": (P, [i, P, sz, i, P]),
+        "msm_shard_info": (i, [P, i, P, P, P]),
         "msm_run": (i, [P, P, P]), "msm_run_partial": (i, [P, P, P]), "msm_finalize": (i, [i, P, i, P]),
         "msm_submit": (ctypes.c_long, [P, P]), "msm_wait": (i, [P, ctypes.c_long, P]),
         "msm_set_option": (i, [P, i, ctypes.c_long]), "msm_get_option": (ctypes.c_long, [P, i]),
@@ -147,7 +151,9 @@ def point_from_words(ws, L32):
 class Context:
     """A set of fixed points resident on `ngpus` devices (msm_context_create)."""
 
-    def __init__(self, curve, points, ngpus: int = 1, n: int | None = None):
+    def __init__(self, curve, points, ngpus: int = 1, n: int | None = None, devices=None):
+        """devices: optional CUDA device per shard (msm_context_create_on; a device may
+        repeat: logical shards on one GPU).  Default: shards on the current device onward."""
         self.curve = curve_id(curve)
         self.L32 = field_words(self.curve)
         self.S = scalar_words(self.curve)
@@ -155,11 +161,24 @@ class Context:
             n = (points.numel() if hasattr(points, "numel") else np.asarray(points).size) // (2 * self.L32)
         self.n = n
         p, keep = _ptr(points, words=n * 2 * self.L32) if n else (None, None)
-        h = lib().msm_context_create(self.curve, p, n, ngpus)
+        if devices is not None:
+            ngpus = len(devices)
+            dv = (ctypes.c_int * ngpus)(*devices)
+            h = lib().msm_context_create_on(self.curve, p, n, ngpus, ctypes.cast(dv, ctypes.c_void_p))
+        else:
+            h = lib().msm_context_create(self.curve, p, n, ngpus)
         if not h:
             raise MSMError(lib().msm_last_error(), "msm_context_create")
         self._h = ctypes.c_void_p(h)
         self.ngpus = ngpus
+
+    def shard_info(self, g: int):
+        """(device, offset, count) of shard g."""
+        d = ctypes.c_int()
+        off = ctypes.c_size_t()
+        cnt = ctypes.c_size_t()
+        _check(lib().msm_shard_info(self._h, g, ctypes.byref(d), ctypes.byref(off), ctypes.byref(cnt)), "msm_shard_info")
+        return d.value, off.value, cnt.value
 
     def close(self):
         if getattr(self, "_h", None):
