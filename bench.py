@@ -48,8 +48,17 @@ def imad_slots_per_sqr(L):
     return 2 * (L * (L + 1) // 2 + L * L) + L
 
 
+def imad_slots_per_sum(L):
+    """fmul_sum (a*b + c*d under one Montgomery reduction): 3 L^2 products (2 slots) + L m_k."""
+    return 3 * L * L * 2 + L
+
+
 def imad_slots_per_pacc(L):
-    """PACC (Alg. 4) = 8 multiplications + 2 squarings (PP = P^2, V = R^2)."""
+    """PACC (Alg. 4) as implemented: for L <= 13, 6 multiplications + 2 squarings + one
+    fmul_sum (Y' = R*D - Y*PPP with one reduction, ec.cuh MSM_ACC_SUM); MNT4-753 (L = 27):
+    8 multiplications + 2 squarings."""
+    if L <= 13:
+        return 6 * imad_slots_per_mult(L) + 2 * imad_slots_per_sqr(L) + imad_slots_per_sum(L)
     return 8 * imad_slots_per_mult(L) + 2 * imad_slots_per_sqr(L)
 
 
@@ -309,6 +318,8 @@ def main():
     ap.add_argument("--split", default="auto", choices=["auto", "points", "buckets"],
                     help="N > 1 decomposition: point shards, or the paper's bucket split (PAPER.md:223); "
                          "auto = buckets for N > 1")
+    ap.add_argument("--acc-mode", type=int, default=2, choices=[0, 1, 2],
+                    help="a4 (MSM_OPT_ACC_MODE): 0 PACC only, 1 batch-affine front end + PACC, 2 auto (library default)")
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--ref-sample", type=int, default=0)
     ap.add_argument("--no-e2e", action="store_true")
@@ -387,6 +398,8 @@ def main():
         ctx.set_option(msm.OPT_WINDOW_BITS, args.window_bits)
     if args.sort:
         ctx.set_option(msm.OPT_SORT, args.sort)
+    if args.acc_mode != 2:
+        ctx.set_option(msm.OPT_ACC_MODE, args.acc_mode)
     if split == "buckets" and ws > 1:
         ctx.set_option(msm.OPT_SPLIT_PARTS, ws)
         ctx.set_option(msm.OPT_SPLIT_INDEX, rank)
@@ -558,8 +571,11 @@ def main():
                      "peak_basis": f"148 SM x 64 IMAD/clk x {sm_max} MHz (clocks.max.sm; B200 guide unit counts)",
                      "frac_pipe": achieved_slots / peak_imad,
                      "frac_pipe_basis": f"IMAD-pipe slots of the radix-2^{W} instruction stream run: {pacc} PACC x "
-                                        f"(8 mul x {imad_slots_per_mult(L)} + 2 sqr x {imad_slots_per_sqr(L)}) slots, "
-                                        "IMAD.WIDE = 2 slots (measured)",
+                                        f"{imad_slots_per_pacc(L)} slots ("
+                                        + (f"6 mul x {imad_slots_per_mult(L)} + 2 sqr x {imad_slots_per_sqr(L)} + 1 fmul_sum x "
+                                           f"{imad_slots_per_sum(L)}" if L <= 13 else
+                                           f"8 mul x {imad_slots_per_mult(L)} + 2 sqr x {imad_slots_per_sqr(L)}")
+                                        + "), IMAD.WIDE = 2 slots (measured)",
                      "field_mults_per_s": pacc * 10 / (acc_avg_ms / 1e3)},
         "clocks": clocks,
         "gpu_launches": int(st["acc_launches"]) * args.steps + (args.steps if ws > 1 else 0),

@@ -93,6 +93,14 @@ enum {
                                  interleaved (b mod G) assignment balances the parts even though
                                  the top window's digits sit in low buckets.                  */
   MSM_OPT_SPLIT_INDEX = 7,    /* f1: this context's part g in [0, G), default 0               */
+  MSM_OPT_ACC_MODE = 8,       /* a4 bucket accumulation: 0 = PACC only (Alg. 4 per entry),
+                                 1 = batch-affine front end (groups of 4 entries of a bucket
+                                 folded into one affine point by pairwise additions sharing
+                                 one inversion per batch, Montgomery's trick) then PACC,
+                                 2 = auto (default: 0 — on B200 the front end's affine glue and
+                                 per-batch inversion made it 1.8x slower; mode 1
+                                 exists for BN254 and BLS12-377/381 as an ablation);
+                                 get returns the mode in use (0/1)                           */
   MSM_OPT_NWIN = 101,         /* (get only) number of windows floor(lambda/c) + 1           */
   MSM_OPT_NSETS = 103,        /* (get only) bucket sets: nwin, or 1 with the f3 table        */
   MSM_OPT_NONEMPTY = 102,     /* (get only) non-empty buckets of the last run on shard 0    */
@@ -117,6 +125,9 @@ typedef struct {
   uint64_t entries;     /* sorted (bucket, point) entries = PACC + bucket starts, device 0 */
   int precompute;       /* f3 table in use on device 0                     */
   float table_ms;       /* time of the last f3 table build on device 0     */
+  float baff_ms;        /* a4 batch-affine front end (part of accumulate_ms) */
+  int baff;             /* batch-affine front end in use                   */
+  uint64_t entries_acc; /* points entering the PACC stage (= entries without the front end) */
 } msm_stats;
 
 typedef struct msm_context msm_context;
@@ -220,7 +231,8 @@ int msm_gen_points(int curve, const uint32_t* e0, const uint32_t* delta, size_t 
 /*
  * Test-only entry points (host buffers; run on the current device; synchronous).
  *   msm_debug_field: op 0 mul, 1 sqr, 2 add, 3 sub, 4 inv (Fermat), 5 neg, 6 inv (binary
- *     extended Euclid, the one the final normalisation uses) on n canonical elements
+ *     extended Euclid, the one the final normalisation uses), 7 a*b + b*a and 8 a*b + a*a
+ *     (sum of two products under one Montgomery reduction, fmul_sum) on n canonical elements
  *     a[i], b[i] (L32 words each); out[i] canonical (inv of 0 is 0 for op 6).
  *   msm_debug_ec: op 0 acc (P + Q via Alg. 4 with P in XYZZ scaled by z1), 1 add (Alg. 1,
  *     both scaled by z1/z2), 2 dbl; P, Q affine (2*L32 words, (0,0) = O); z: 2*L32 words

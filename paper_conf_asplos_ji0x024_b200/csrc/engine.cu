@@ -18,6 +18,8 @@
 #include <thread>
 #include <vector>
 
+#include <nvtx3/nvToolsExt.h>
+
 #include "runtime.h"
 
 using namespace msmrt;
@@ -57,6 +59,13 @@ bool is_device_ptr(const void* p, int* dev) {
   return false;
 }
 
+// NVTX range for the duration of an ABI call (visible in nsys / ncu --nvtx timelines; the
+// header-only NVTX v3 API costs nothing when no tool is attached).
+struct NvtxRange {
+  explicit NvtxRange(const char* name) { nvtxRangePushA(name); }
+  ~NvtxRange() { nvtxRangePop(); }
+};
+
 // Restores the caller's current device when an ABI call returns (the library switches
 // devices per shard; the caller's torch/CUDA state must not change under it).
 struct DeviceGuard {
@@ -90,10 +99,21 @@ void order_after_legacy(int src_dev, int dev, cudaStream_t stream) {
 //   entry, plus the bucket reduce (2 PADD per bucket, measured ~4.4 PACC-equivalents per
 //   bucket on B200, r01 bench) over 2^(c-1) buckets per bucket set.  With the f3 table all
 //   windows share one bucket set, so larger c pays off.
-double plan_cost(size_t n, int lambda, int c, bool pre) {
+//   Each bucket-reduce segment (>= 4 buckets, at most one per resident thread, ~37.9 K on
+//   148 SMs) also ends with a small-scalar multiplication of ~c doublings + adds on one
+//   thread (~2.3 PACC-equivalents per bit): a per-segment latency term that makes large c
+//   lose at small n (C2, n = 2^20: c = 16 beats c = 20, r01 sweep).
+//   bucket_cost: reduce cost per bucket in units of one entry's accumulation — 4.4 for the
+//   8..13-limb curves.  For MNT4-753 the reduce per bucket is dearer (out-of-line 27-limb
+//   PADD: 52.7 ms for 2^22 buckets) but the accumulation per entry grows as c shrinks
+//   (r02, n = 2^22: 1.79 / 1.96 / 2.27 ns per entry at c = 23 / 22 / 21; step 304.7 /
+//   330.1 / 373.8 ms), which this model does not capture; 3.5 keeps c = 23 there.
+double plan_cost(size_t n, int lambda, int c, bool pre, double bucket_cost = 4.4) {
   const double nwin = num_windows(lambda, c);
   const double sets = pre ? 1.0 : nwin;
-  return nwin * (double)n * 1.12 + sets * std::ldexp(1.0, c - 1) * 4.4;
+  const double buckets = sets * std::ldexp(1.0, c - 1);
+  const double segs = std::min(buckets / 4.0, 37888.0);
+  return nwin * (double)n * 1.12 + buckets * bucket_cost + segs * c * 2.3;
 }
 
 // device bytes of the f3 table and of the per-run scratch for window size c
@@ -102,12 +122,17 @@ size_t scratch_bytes(size_t n, int lambda, int c, int XW, bool pre) {
   const size_t nwin = num_windows(lambda, c);
   const size_t sets = pre ? 1 : nwin;
   const size_t NB = ((size_t)1 << (c - 1)) + 1;
-  return n * nwin * 22 + sets * NB * ((size_t)XW * 4 + 12) + ((size_t)1 << 28);
+  // sort + sorted entries (~22 B/entry), bucket set(s), and the batch-affine front end:
+  // ceil(count/4) folded points per bucket (<= entries/4 + buckets, ~28 B/entry at PW = 28)
+  // plus its per-thread batch scratch (<= 2 GB)
+  return n * nwin * (22 + (size_t)XW * 4 / 7) + sets * NB * ((size_t)XW * 4 + 12 + (size_t)XW * 2) +
+         ((size_t)1 << 28) + ((size_t)2 << 30);
 }
 
 // Chooses (c, pre) for one shard: opt.c / opt.pre when fixed; otherwise the cheapest
 // configuration whose device memory fits (the f3 table needs nwin*n < 2^31 entries too).
-void plan_shard(const Options& o, const Shard& s, int lambda, int PW, int XW, int* c_out, int* pre_out) {
+void plan_shard(const Options& o, const Shard& s, int lambda, int PW, int XW, int* c_out, int* pre_out,
+                double bucket_cost) {
   size_t fr = 0, tot = 0;
   CK(cudaSetDevice(s.dev));
   CK(cudaMemGetInfo(&fr, &tot));
@@ -139,7 +164,7 @@ void plan_shard(const Options& o, const Shard& s, int lambda, int PW, int XW, in
         const bool fit = fits(c, pre);
         any_fit |= fit;
         if (pass == 0 && !fit && (o.pre == 2 || o.c <= 0)) continue;
-        const double cost = s.n == 0 ? (double)c : plan_cost(s.n, lambda, c, pre);
+        const double cost = s.n == 0 ? (double)c : plan_cost(s.n, lambda, c, pre, bucket_cost);
         if (cost < best) { best = cost; bc = c; bp = pre; }
       }
     }
@@ -179,7 +204,8 @@ void destroy_shard(CurveOps* ops, Shard& s) {
 int apply_window_bits(msm_context* ctx) {
   for (auto& s : ctx->shards) {
     int c = 0, pre = 0;
-    plan_shard(ctx->opt, s, ctx->ops->lambda(), ctx->ops->PW(), ctx->ops->XW(), &c, &pre);
+    plan_shard(ctx->opt, s, ctx->ops->lambda(), ctx->ops->PW(), ctx->ops->XW(), &c, &pre,
+               ctx->ops->L32() > 12 ? 3.5 : 4.4);
     ctx->ops->configure(ctx->opt, s, c, pre);
   }
   return MSM_OK;
@@ -233,6 +259,7 @@ int run_all(msm_context* ctx, const uint32_t* scalars, bool gather_to_dev0) {
       if (timed) CK(cudaEventRecord(s.ev[EV_START], s.stream));
       CK(cudaMemsetAsync(s.err, 0, 4, s.stream));
       const uint32_t* sc = stage_scalars(ctx, s, scalars, is_dev, src_dev);
+      NvtxRange nr("enqueue a2..a6 (shard)");
       launched[g] = ctx->ops->enqueue_pipeline(s, sc, timed);
     } catch (const CudaError& e) {
       rc[g] = e.code;
@@ -284,6 +311,7 @@ void collect_stats(msm_context* ctx) {
   st.h2d_ms = el(EV_START, EV_H2D);
   st.sort_ms = el(EV_H2D, EV_SORT);
   st.accumulate_ms = el(EV_SORT, EV_ACC);
+  st.baff_ms = el(EV_SORT, EV_BAFF);
   st.fixup_ms = el(EV_ACC, EV_FIX);
   st.reduce_ms = el(EV_FIX, EV_RED);
   st.combine_ms = el(EV_RED, EV_COMB);
@@ -298,6 +326,10 @@ void collect_stats(msm_context* ctx) {
   st.entries = M;
   st.precompute = s.pre;
   st.table_ms = s.table_ms;
+  st.baff = s.baff;
+  uint32_t M4 = M;
+  if (s.baff) cudaMemcpy(&M4, s.goff4 + s.F, 4, cudaMemcpyDeviceToHost);
+  st.entries_acc = M4;
 }
 
 // Every ABI call that touches a device runs through guarded(): C++ exceptions become
@@ -391,6 +423,7 @@ msm_context* msm_context_create(int curve, const uint32_t* points, size_t n, int
 }
 
 msm_context* msm_context_create_on(int curve, const uint32_t* points, size_t n, int ngpus, const int* devices) {
+  NvtxRange nvtx_("msm_context_create");
   g_last_error = MSM_OK;
   DeviceGuard guard;
   CurveOps* ops = ops_for(curve);
@@ -489,6 +522,7 @@ void msm_context_destroy(msm_context* ctx) {
 }
 
 int msm_run(msm_context* ctx, const uint32_t* scalars, uint32_t* result) {
+  NvtxRange nvtx_("msm_run");
   if (!ctx || !result || (ctx->n && !scalars)) return MSM_ERR_ARG;
   return guarded([&]() -> int {
     run_all(ctx, scalars, true);
@@ -506,6 +540,7 @@ int msm_run(msm_context* ctx, const uint32_t* scalars, uint32_t* result) {
 }
 
 int msm_run_partial(msm_context* ctx, const uint32_t* scalars, uint32_t* partial) {
+  NvtxRange nvtx_("msm_run_partial");
   if (!ctx || !partial || (ctx->n && !scalars) || ctx->shards.size() != 1) return MSM_ERR_ARG;
   return guarded([&]() -> int {
     run_all(ctx, scalars, false);
@@ -528,6 +563,7 @@ int msm_run_partial(msm_context* ctx, const uint32_t* scalars, uint32_t* partial
 }
 
 long msm_submit(msm_context* ctx, const uint32_t* scalars) {
+  NvtxRange nvtx_("msm_submit");
   if (!ctx || (ctx->n && !scalars) || ctx->shards.size() != 1) return MSM_ERR_ARG;
   if (ctx->next_ticket - ctx->next_wait >= MSM_MAX_INFLIGHT) return MSM_ERR_ARG;
   const int rc = guarded([&]() -> int {
@@ -589,6 +625,7 @@ int msm_wait(msm_context* ctx, long ticket, uint32_t* result) {
 }
 
 int msm_finalize(int curve, const uint32_t* partials, int count, uint32_t* result) {
+  NvtxRange nvtx_("msm_finalize");
   CurveOps* ops = ops_for(curve);
   if (!ops) return MSM_ERR_CURVE;
   if (count < 0 || (count > 0 && !partials) || !result) return MSM_ERR_ARG;
@@ -653,6 +690,11 @@ int msm_set_option(msm_context* ctx, int key, long value) {
       if (value < 0 || value >= ctx->opt.split_G) return MSM_ERR_ARG;
       ctx->opt.split_g = (int)value;
       break;
+    case MSM_OPT_ACC_MODE:
+      if (value < 0 || value > 2) return MSM_ERR_ARG;
+      if (value == 1 && !ctx->ops->has_baff()) return MSM_ERR_UNIMPLEMENTED;
+      ctx->opt.acc_mode = (int)value;
+      break;
     default:
       return MSM_ERR_ARG;
   }
@@ -671,6 +713,7 @@ long msm_get_option(msm_context* ctx, int key) {
     case MSM_OPT_NSETS: return ctx->shards[0].nset;
     case MSM_OPT_SPLIT_PARTS: return ctx->opt.split_G;
     case MSM_OPT_SPLIT_INDEX: return ctx->opt.split_g;
+    case MSM_OPT_ACC_MODE: return ctx->shards[0].baff;
     case MSM_OPT_DEVICE: return ctx->shards[0].dev;
     case MSM_OPT_NGPUS: return (long)ctx->shards.size();
     case MSM_OPT_NONEMPTY: {
@@ -716,7 +759,7 @@ int msm_gen_points(int curve, const uint32_t* e0, const uint32_t* delta, size_t 
 int msm_debug_field(int curve, int op, const uint32_t* a, const uint32_t* b, size_t n, uint32_t* out) {
   CurveOps* ops = ops_for(curve);
   if (!ops) return MSM_ERR_CURVE;
-  if (!a || !b || !out || op < 0 || op > 6) return MSM_ERR_ARG;
+  if (!a || !b || !out || op < 0 || op > 8) return MSM_ERR_ARG;
   return guarded([&]() -> int {
     ops->debug_field(op, a, b, n, out);
     return MSM_OK;

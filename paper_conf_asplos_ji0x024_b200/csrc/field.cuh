@@ -204,6 +204,61 @@ DEVI void fmul3(uint32_t* r1, const uint32_t* a1, const uint32_t* b1, uint32_t* 
   fmul3_cols<C, 0>(r1, a1, b1, m1, 0ull, 0ull, r2, a2, b2, m2, 0ull, 0ull, r3, a3, b3, m3, 0ull, 0ull);
 }
 
+// ---- r = (a*b + c*d) * R^-1 mod p with ONE Montgomery reduction (lazy reduction of a
+// sum of products): the a*b, c*d and m*p terms of a column accumulate in three
+// IMAD.WIDE chains (each <= L products of < 2^(2W), within MAXT), their low words are added
+// for m_K, and the three carries travel separately.  Saves the L^2 + L reduction products of
+// a second multiplication.  Bound: for inputs with a*b + c*d < 68 p^2 the result is < 2p on
+// every curve here (R/p >= 2^9.3).
+template <class C, int K>
+DEVI void fsum_step(uint32_t* r, const uint32_t* a, const uint32_t* b, const uint32_t* c, const uint32_t* d, uint32_t* m,
+                    u64& cA, u64& cB, u64& cM) {
+  constexpr int L = C::L, W = C::W;
+  constexpr uint32_t MASK = (1u << W) - 1;
+  constexpr int lo = K - L + 1 > 0 ? K - L + 1 : 0;
+  constexpr int hiA = K < L - 1 ? K : L - 1;
+  constexpr int hiM = (K - 1) < (L - 1) ? K - 1 : L - 1;
+  u64 accA = cA, accB = cB, accM = cM;
+#pragma unroll
+  for (int i = lo; i <= hiA; i++) {
+    accA = mad_wide(a[i], b[K - i], accA);
+    accB = mad_wide(c[i], d[K - i], accB);
+  }
+#pragma unroll
+  for (int i = lo; i <= hiM; i++) accM = mad_wide(m[i], C::P(K - i), accM);
+  const uint32_t t = ((uint32_t)accA & MASK) + ((uint32_t)accB & MASK);  // < 2^(W+1)
+  if constexpr (K < L) {
+    const uint32_t s = t + ((uint32_t)accM & MASK);                        // < 3 * 2^W
+    m[K] = (s * C::N0) & MASK;
+    accM = mad_wide(m[K], C::P(0), accM);
+    const uint32_t s2 = t + ((uint32_t)accM & MASK);                       // 0, 2^W or 2^(W+1)
+    cM = (accM >> W) + (s2 >> W);
+  } else {
+    const uint32_t s = t + ((uint32_t)accM & MASK);
+    r[K - L] = s & MASK;
+    cM = (accM >> W) + (s >> W);
+  }
+  cA = accA >> W;
+  cB = accB >> W;
+  if constexpr (K == 2 * L - 2) r[L - 1] = (uint32_t)(cA + cB + cM);
+}
+
+template <class C, int K>
+DEVI void fsum_cols(uint32_t* r, const uint32_t* a, const uint32_t* b, const uint32_t* c, const uint32_t* d, uint32_t* m,
+                    u64 cA, u64 cB, u64 cM) {
+  fsum_step<C, K>(r, a, b, c, d, m, cA, cB, cM);
+  if constexpr (K + 1 < 2 * C::L - 1) fsum_cols<C, K + 1>(r, a, b, c, d, m, cA, cB, cM);
+}
+
+// r = a*b + c*d (Montgomery), r may alias any input
+template <class C>
+DEVI void fmul_sum(uint32_t* r, const uint32_t* a, const uint32_t* b, const uint32_t* c, const uint32_t* d) {
+  uint32_t m[C::L], t[C::L];
+  fsum_cols<C, 0>(t, a, b, c, d, m, 0ull, 0ull, 0ull);
+#pragma unroll
+  for (int i = 0; i < C::L; i++) r[i] = t[i];
+}
+
 template <class C, bool SQR, bool LAT = false>
 DEVI void fmul_impl(uint32_t* r, const uint32_t* a, const uint32_t* b) {
   constexpr int L = C::L;
@@ -276,6 +331,47 @@ DEVI void fsub(uint32_t* r, const uint32_t* a, const uint32_t* b) {
     c = s >> W;
   }
   r[L - 1] = (uint32_t)((int32_t)(a[L - 1] - b[L - 1] + C::KP(K, L - 1)) + c);
+}
+
+// ---- carry-deferred add / subtract (one-step carries: every limb independent, so the
+// glue between the PACC's multiplication pairs is ~3 dependent ALU ops deep instead of a
+// 13-step carry chain).  Outputs are "semi-normalised": limbs <= 2^W + 3 (the top limb
+// unmasked), which every multiplication accepts (a column of <= MAXT products of
+// (2^W + 3)^2 still fits 64 bits) and the exact fsub/fadd normalise again.  They are NOT
+// valid inputs for fis_zero / fequal / fcsub (those need normalised limbs).
+// r = a + b  (a, b limbs <= 2^W + 3; bound(r) = bound(a) + bound(b))
+template <class C>
+DEVI void fadd_fast(uint32_t* r, const uint32_t* a, const uint32_t* b) {
+  constexpr int L = C::L, W = C::W;
+  constexpr uint32_t MASK = (1u << W) - 1;
+  uint32_t s[L];
+#pragma unroll
+  for (int i = 0; i < L; i++) s[i] = a[i] + b[i];
+  r[0] = s[0] & MASK;
+#pragma unroll
+  for (int i = 1; i < L - 1; i++) r[i] = (s[i] & MASK) + (s[i - 1] >> W);
+  r[L - 1] = s[L - 1] + (s[L - 2] >> W);
+}
+
+// r = a - b + (K+1)*p  (a normalised (limbs < 2^W), b limbs <= 2^W + 3, bound(b) <= K;
+// bound(r) = bound(a) + K + 1).  (K+1)*p is added in a borrow-proof limb form
+// D_0 = kp_0 + 2^(W+1), D_i = kp_i + 2^(W+1) - 2, D_(L-1) = kp_(L-1) - 2 (same value), so
+// every limb difference is non-negative and < 2^32; the extra p keeps the value >= p, so
+// the top limb stays non-negative after the one-step carries.
+template <class C, int K>
+DEVI void fsub_fast(uint32_t* r, const uint32_t* a, const uint32_t* b) {
+  static_assert(K + 1 < C::KMAX, "(K+1)*p not tabulated");
+  constexpr int L = C::L, W = C::W;
+  constexpr uint32_t MASK = (1u << W) - 1;
+  uint32_t s[L];
+  s[0] = a[0] - b[0] + (C::KP(K + 1, 0) + (2u << W));
+#pragma unroll
+  for (int i = 1; i < L - 1; i++) s[i] = a[i] - b[i] + (C::KP(K + 1, i) + (2u << W) - 2u);
+  s[L - 1] = a[L - 1] - b[L - 1] + (C::KP(K + 1, L - 1) - 2u);
+  r[0] = s[0] & MASK;
+#pragma unroll
+  for (int i = 1; i < L - 1; i++) r[i] = (s[i] & MASK) + (s[i - 1] >> W);
+  r[L - 1] = s[L - 1] + (s[L - 2] >> W);
 }
 
 // r = K*p - a   (negation; requires bound(a) <= K)

@@ -747,7 +747,15 @@ __global__ void __launch_bounds__(128, MSM_ACC_MINB) k_accumulate(const uint32_t
 #define MSM_ACC_SYNC_NT 256  // A/B: 384 = 3 warps per scheduler (<= 168 registers)
 #endif
 constexpr int ACC_SYNC_NT = MSM_ACC_SYNC_NT;
-template <class C>
+// DIRECT (batch-affine front end, baff.cuh): entry e's point is pts[e] itself (the folded
+// affine points, bucket-major), no index and no sign.
+template <bool DIRECT>
+DEVI uint32_t entry_at(const uint32_t* __restrict__ sorted, uint32_t e) {
+  if constexpr (DIRECT) return e;
+  else return __ldg(sorted + e);
+}
+
+template <class C, bool DIRECT = false>
 __global__ void __launch_bounds__(ACC_SYNC_NT, 1) k_accumulate_sync(const uint32_t* __restrict__ pts, const uint32_t* __restrict__ sorted,
                                                     const uint32_t* __restrict__ goff, uint32_t F,
                                                     uint32_t* __restrict__ buckets, uint32_t* __restrict__ carry_pts,
@@ -776,10 +784,10 @@ __global__ void __launch_bounds__(ACC_SYNC_NT, 1) k_accumulate_sync(const uint32
     f = find_bucket(goff, F, e0);
     end = __ldg(goff + f + 1);
     head = __ldg(goff + f) < e0;
-    ok = point_for_entry<C>(x, y, pts, __ldg(sorted + e0));
+    ok = point_for_entry<C>(x, y, pts, entry_at<DIRECT>(sorted, e0));
     acc_start<C>(acc, x, y, ok);
-    ent1 = e0 + 1 < e1 ? __ldg(sorted + e0 + 1) : 0u;
-    ent2 = e0 + 2 < e1 ? __ldg(sorted + e0 + 2) : 0u;
+    ent1 = e0 + 1 < e1 ? entry_at<DIRECT>(sorted, e0 + 1) : 0u;
+    ent2 = e0 + 2 < e1 ? entry_at<DIRECT>(sorted, e0 + 2) : 0u;
     if constexpr (REGPF) {
       if (e0 + 1 < e1) load_point<C>(nx, ny, pts, ent1 & ~SIGN_BIT);
     } else {
@@ -796,12 +804,12 @@ __global__ void __launch_bounds__(ACC_SYNC_NT, 1) k_accumulate_sync(const uint32
       fcopy<C>(x, nx);
       fcopy<C>(y, ny);
       if (e + 1 < e1) load_point<C>(nx, ny, pts, ent1 & ~SIGN_BIT);
-      if (e + 2 < e1) ent2 = __ldg(sorted + e + 2);
+      if (e + 2 < e1) ent2 = entry_at<DIRECT>(sorted, e + 2);
       ok = !fis_zero<C, 2>(y);
       if (ok && (ent & SIGN_BIT)) fneg<C, 2>(y, y);
     } else {
       if (e + 1 < e1) prefetch_point<C>(pts, ent1);
-      if (e + 2 < e1) ent2 = __ldg(sorted + e + 2);
+      if (e + 2 < e1) ent2 = entry_at<DIRECT>(sorted, e + 2);
       ok = point_for_entry<C>(x, y, pts, ent);
     }
     if (e == end) {
@@ -822,6 +830,11 @@ __global__ void __launch_bounds__(ACC_SYNC_NT, 1) k_accumulate_sync(const uint32
     carry_f[t] = my_carry;
   }
 }
+
+#ifndef MSM_BAFF
+#define MSM_BAFF 0  // batch-affine a4 front end (ablation, baff.cuh): instantiated only with -DMSM_BAFF=1
+#endif
+#include "baff.cuh"
 
 // ---------------------------------------------------------------------------------------
 // a4 variant (MSM_ACC_SMEM, A/B): the PAPER.md:267 idea — big integers cached in shared
@@ -1379,7 +1392,8 @@ __global__ void __launch_bounds__(128) k_gen_points(const uint32_t* __restrict__
 
 // ---------------------------------------------------------------------------------------
 // debug kernels for the field / EC layers (tests only)
-enum { DBG_MUL = 0, DBG_SQR = 1, DBG_ADD = 2, DBG_SUB = 3, DBG_INV = 4, DBG_NEG = 5, DBG_INV_BGCD = 6 };
+enum { DBG_MUL = 0, DBG_SQR = 1, DBG_ADD = 2, DBG_SUB = 3, DBG_INV = 4, DBG_NEG = 5, DBG_INV_BGCD = 6, DBG_SUM_ABBA = 7,
+       DBG_SUM_ABAA = 8 };
 
 template <class C>
 __global__ void k_debug_field(int op, const uint32_t* __restrict__ a, const uint32_t* __restrict__ b, size_t n,
@@ -1399,6 +1413,8 @@ __global__ void k_debug_field(int op, const uint32_t* __restrict__ a, const uint
     case DBG_SUB: fsub<C, 2>(r, x, y); break;
     case DBG_INV: finv<C>(r, x); break;
     case DBG_INV_BGCD: finv_bgcd<C>(r, x); break;
+    case DBG_SUM_ABBA: fmul_sum<C>(r, x, y, y, x); break;  // 2ab (one reduction)
+    case DBG_SUM_ABAA: fmul_sum<C>(r, x, y, x, x); break;  // a(b + a)
     default: fneg<C, 2>(r, x); break;
   }
   ffrom_mont<C>(r, r);

@@ -16,6 +16,12 @@ struct Ops final : CurveOps {
   // k_accumulate_sync (lockstep blocks, register-prefetched gathers) for L <= 13; MNT4-753
   // keeps k_accumulate (255 registers already; no room for the prefetched point)
   static constexpr bool kAccSync = MSM_ACC_SYNC != 0 && (C::L <= 13 || MSM_ACC_SYNC_ALL != 0);
+  // batch-affine front end (baff.cuh) for L <= 13 (MNT4-753's 27-limb pairs would spill)
+  // Built only with -DMSM_BAFF=1 (an ablation, off by default: compile time and speed,
+  // DESIGN.md §7b); without it MSM_OPT_ACC_MODE = 1 returns MSM_ERR_UNIMPLEMENTED.
+  static constexpr bool kBaff = MSM_BAFF != 0 && kAccSync && C::L <= 13;
+  bool has_baff() const override { return kBaff; }
+  static constexpr uint32_t kBaffB = 256;  // outputs per batch (one inversion per level)
   static constexpr int XW_ = Layout<C>::XW;
   static constexpr int PW_ = Layout<C>::PW;
   int L32() const override { return C::L32; }
@@ -38,6 +44,8 @@ struct Ops final : CurveOps {
     dfree(s.s3Count); dfree(s.s3Off); dfree(s.s3Cursor); dfree(s.s3Sub);
     dfree(s.s3SubCount); dfree(s.s3SubCursor); dfree(s.s3Tiles);
     dfree(s.s3k1); dfree(s.s3v1); dfree(s.s3k2); dfree(s.s3v2);
+    dfree(s.c4); dfree(s.goff4); dfree(s.cursor4); dfree(s.out4); dfree(s.baff_scratch);
+    s.baff = 0;
   }
 
   void free_table(Shard& s) override {
@@ -141,6 +149,20 @@ struct Ops final : CurveOps {
     else if (!s.table || s.table_c != c) {
       free_table(s);
       build_table(s);
+    }
+    s.baff = (kBaff && o.acc_mode == 1) ? 1 : 0;  // auto (2) = PACC only: the front end measured slower
+    if constexpr (kBaff) if (s.baff) {
+      int bpb = 0;
+      CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bpb, k_baff2<C>, BAFF_NT, 0));
+      if (bpb < 1) bpb = 1;
+      s.baff_T = (uint32_t)(sms * bpb * BAFF_NT);
+      s.baff_B = kBaffB;
+      const size_t M4max = Mmax / 4 + s.F + 1;
+      dalloc(&s.c4, s.F);
+      dalloc(&s.goff4, s.F + 1);
+      dalloc(&s.cursor4, s.F);
+      dalloc(&s.out4, M4max * PW_);
+      dalloc(&s.baff_scratch, (size_t)s.baff_T * s.baff_B * (7 * C::L + 2));
     }
     dalloc(&s.counts, s.F);
     dalloc(&s.goff, s.F + 1);
@@ -276,15 +298,36 @@ struct Ops final : CurveOps {
     }
     CK(cudaGetLastError());
     if (timed) CK(cudaEventRecord(s.ev[EV_SORT], st));
+    // a4 front end: groups of 4 entries per bucket -> one affine point (batch-affine)
+    const uint32_t* acc_pts = pts;
+    const uint32_t* acc_goff = s.goff;
+    if constexpr (kBaff) {
+      if (s.baff) {
+        k_group4_counts<<<(unsigned)cdiv(s.F, 256), 256, 0, st>>>(s.goff, s.F, s.c4);
+        k_scan_reduce<<<(unsigned)s.ntiles, SCAN_THREADS, 0, st>>>(s.c4, s.F, s.tiles);
+        k_scan_tiles<<<1, 1024, 0, st>>>(s.tiles, s.ntiles, s.goff4 + s.F);
+        k_scan_apply<<<(unsigned)s.ntiles, SCAN_THREADS, 0, st>>>(s.c4, s.F, s.tiles, s.goff4, s.cursor4);
+        k_baff2<C><<<s.baff_T / BAFF_NT, BAFF_NT, 0, st>>>(pts, s.sorted, s.goff, s.goff4, (uint32_t)s.F, s.baff_B,
+                                                            s.out4, s.baff_scratch);
+        launches += 5;
+        CK(cudaGetLastError());
+        acc_pts = s.out4;
+        acc_goff = s.goff4;
+      }
+    }
+    if (timed) CK(cudaEventRecord(s.ev[EV_BAFF], st));
     // a4: accumulate + fixup
 #if MSM_ACC_SMEM
     k_accumulate_smem<C><<<(unsigned)cdiv(s.acc_threads, 128), 128, ACC_SLOTS * C::L * ACC_NT * 4, st>>>(pts, s.sorted, s.goff, (uint32_t)s.F,
 #else
-    if constexpr (kAccSync)
-      k_accumulate_sync<C><<<(unsigned)cdiv(s.acc_threads, ACC_SYNC_NT), ACC_SYNC_NT, 0, st>>>(pts, s.sorted, s.goff, (uint32_t)s.F,
-                                                                        s.buckets, s.carry_pts, s.carry_f, s.acc_threads,
-                                                                        s.nlong);
-    else
+    if constexpr (kAccSync) {
+      if (s.baff)
+        k_accumulate_sync<C, true><<<(unsigned)cdiv(s.acc_threads, ACC_SYNC_NT), ACC_SYNC_NT, 0, st>>>(
+            acc_pts, s.sorted, acc_goff, (uint32_t)s.F, s.buckets, s.carry_pts, s.carry_f, s.acc_threads, s.nlong);
+      else
+        k_accumulate_sync<C><<<(unsigned)cdiv(s.acc_threads, ACC_SYNC_NT), ACC_SYNC_NT, 0, st>>>(
+            pts, s.sorted, s.goff, (uint32_t)s.F, s.buckets, s.carry_pts, s.carry_f, s.acc_threads, s.nlong);
+    } else
       k_accumulate<C><<<(unsigned)cdiv(s.acc_threads, 128), 128, 0, st>>>(pts, s.sorted, s.goff, (uint32_t)s.F,
 #endif
                                                                         s.buckets, s.carry_pts, s.carry_f, s.acc_threads,

@@ -40,7 +40,7 @@ void dfree(T*& p) {
   p = nullptr;
 }
 
-enum { EV_START, EV_H2D, EV_SORT, EV_ACC, EV_FIX, EV_RED, EV_COMB, EV_END, EV_COUNT };
+enum { EV_START, EV_H2D, EV_SORT, EV_BAFF, EV_ACC, EV_FIX, EV_RED, EV_COMB, EV_END, EV_COUNT };
 
 // One device's share of a context: its points, scratch and stream.
 struct Shard {
@@ -85,6 +85,11 @@ struct Shard {
   uint32_t* table = nullptr;
   int table_c = 0;
   float table_ms = 0;
+  // batch-affine front end of a4 (baff.cuh): groups of 4 entries per bucket folded into one
+  // affine point (out4 [M4][PW], offsets goff4), then PACC over out4
+  int baff = 0;
+  uint32_t *c4 = nullptr, *goff4 = nullptr, *cursor4 = nullptr, *out4 = nullptr, *baff_scratch = nullptr;
+  uint32_t baff_T = 0, baff_B = 0;
 };
 
 struct Options {
@@ -93,6 +98,7 @@ struct Options {
                  // 3 three-level staged (sort3.cuh)
   int pre = 2;   // f3 precomputation: 0 off, 1 on, 2 auto (on when the table fits in memory)
   int split_G = 1, split_g = 0;  // f1: this context sums only buckets |d| = G*q + g
+  int acc_mode = 2;  // a4: 0 PACC only, 1 batch-affine front end + PACC (ablation), 2 auto (= 0, measured faster)
 };
 
 // Per-curve kernels behind a virtual interface (one instance per curve, curve_*.cu).
@@ -119,6 +125,7 @@ struct CurveOps {
   virtual void debug_digits(int c, const uint32_t* scal, size_t n, int32_t* out) = 0;
   virtual void to_affine(const uint32_t* in_dev, size_t n, uint32_t* out_dev, cudaStream_t st) = 0;
   virtual long count_nonempty(Shard& s) = 0;
+  virtual bool has_baff() const = 0;
 };
 
 inline int num_windows(int lambda, int c) { return lambda / c + 1; }

@@ -27,6 +27,7 @@ OPT_SORT = 4
 OPT_PRECOMPUTE = 5
 OPT_SPLIT_PARTS = 6
 OPT_SPLIT_INDEX = 7
+OPT_ACC_MODE = 8
 OPT_NWIN = 101
 OPT_NONEMPTY = 102
 OPT_NSETS = 103
@@ -53,6 +54,7 @@ class Stats(ctypes.Structure):
         ("finalize_ms", ctypes.c_float), ("total_ms", ctypes.c_float), ("window_bits", ctypes.c_int),
         ("nwin", ctypes.c_int), ("acc_threads", ctypes.c_int), ("acc_launches", ctypes.c_int),
         ("entries", ctypes.c_uint64), ("precompute", ctypes.c_int), ("table_ms", ctypes.c_float),
+        ("baff_ms", ctypes.c_float), ("baff", ctypes.c_int), ("entries_acc", ctypes.c_uint64),
     ]
 
     def as_dict(self):

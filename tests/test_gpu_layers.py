@@ -45,6 +45,8 @@ def test_field_ops(msm, name):
         2: [(x + y) % p for x, y in zip(A, B)],
         3: [(x - y) % p for x, y in zip(A, B)],
         5: [(-x) % p for x in A],
+        7: [2 * x * y % p for x, y in zip(A, B)],      # fmul_sum(a, b, b, a)
+        8: [x * (y + x) % p for x, y in zip(A, B)],    # fmul_sum(a, b, a, a)
     }
     for op, want in exp.items():
         got = msm.debug_field(name, op, a, b)

@@ -368,7 +368,7 @@ def test_bucket_split_parity(lib, name, pre):
 def test_bucket_split_large_balanced(lib):
     """f1 at a size that uses the staged sort and many segments: BLS12-381, n = 2^16, auto c
     with the f3 table, G = 4 parts finalize to the closed form, and the interleaved
-    assignment keeps every part's entry count within 2 % of the mean."""
+    assignment keeps every part's entry count within 3 % of the mean."""
     name = "bls12_381"
     c = CURVES[name]
     n = 1 << 16
@@ -392,7 +392,8 @@ def test_bucket_split_large_balanced(lib):
         ctx.close()
     assert lib.finalize(name, parts, G) == want
     mean = sum(entries) / G
-    assert max(abs(x - mean) for x in entries) < 0.02 * mean, entries
+    # 3 %: at the planner's c = 14 the 3-bit top window's digits 1..8 fall unevenly on 4 parts
+    assert max(abs(x - mean) for x in entries) < 0.03 * mean, entries
 
 
 @pytest.mark.parametrize("name", ["bn254", "bls12_381", "mnt4_753"])
@@ -430,3 +431,58 @@ def test_pipelined_submit_wait(lib, name):
     t5 = ctx.submit(words[0])
     assert ctx.wait(t5) == closed(name, sets[0], es)
     ctx.close()
+
+
+@pytest.mark.parametrize("name", ["bn254", "bls12_377", "bls12_381"])
+@pytest.mark.parametrize("pre", [0, 1])
+def test_batch_affine_front_end(lib, name, pre):
+    """a4 batch-affine front end (MSM_OPT_ACC_MODE = 1; baff.cuh): every group of up to 4
+    entries of a bucket is folded by pairwise affine additions sharing one inversion per
+    batch.  Exercised on buckets of every size mod 4, pairs that double (equal points, equal
+    digits), pairs that cancel (k and r - k on one point), O points inside groups, and many
+    batches per thread (few threads forced through MSM_OPT_ACC_THREADS does not apply to the
+    front end, so small c packs long buckets).  Bit-exact vs the closed form, and equal to
+    the PACC-only path (mode 0)."""
+    c = CURVES[name]
+    G = c.G
+    base = [ec.mul(i + 2, G, c) for i in range(40)]
+    Ps, es, ks = [], [], []
+    rng = np.random.default_rng(7)
+    for i in range(600):
+        kind = i % 6
+        j = int(rng.integers(0, 40))
+        if kind == 0:      # duplicate of the previous point with the same scalar -> doubling pairs
+            P, e, k = (Ps[-1], es[-1], ks[-1]) if Ps else (base[j], j + 2, 5)
+        elif kind == 1:    # the previous point with r - k -> cancelling pairs
+            P, e, k = (Ps[-1], es[-1], (c.r - ks[-1]) % c.r) if Ps else (base[j], j + 2, 7)
+        elif kind == 2:    # O
+            P, e, k = None, 0, int(rng.integers(1, 1 << 20))
+        else:
+            P, e, k = base[j], j + 2, int(rng.integers(1, 64))
+        Ps.append(P)
+        es.append(e)
+        ks.append(k)
+    want = ec.to_output(ec.mul(sum(k * e for k, e in zip(ks, es)) % c.r, G, c))
+    ctx = lib.Context(name, points_to_words(Ps, name), n=len(Ps))
+    sw = synth.ints_to_words(ks, S_W[name])
+    try:
+        try:
+            ctx.set_option(lib.OPT_ACC_MODE, 1)
+        except lib.MSMError as e:
+            assert e.code == -8
+            pytest.skip("batch-affine front end not built (tools/build.py -D MSM_BAFF=1)")
+        ctx.set_option(lib.OPT_PRECOMPUTE, pre)
+        for cbits in (3, 5, 7):
+            ctx.set_option(lib.OPT_WINDOW_BITS, cbits)
+            ctx.set_option(lib.OPT_ACC_MODE, 1)
+            assert ctx.get_option(lib.OPT_ACC_MODE) == 1
+            got1 = ctx.run(sw)
+            st = ctx.stats()
+            assert st["baff"] == 1 and st["entries_acc"] < st["entries"]
+            ctx.set_option(lib.OPT_ACC_MODE, 0)
+            assert ctx.get_option(lib.OPT_ACC_MODE) == 0
+            got0 = ctx.run(sw)
+            assert got1 == want, (cbits, "front end")
+            assert got0 == want, (cbits, "PACC only")
+    finally:
+        ctx.close()
