@@ -54,12 +54,9 @@ def imad_slots_per_sum(L):
 
 
 def imad_slots_per_pacc(L):
-    """PACC (Alg. 4) as implemented: for L <= 13, 6 multiplications + 2 squarings + one
-    fmul_sum (Y' = R*D - Y*PPP with one reduction, ec.cuh MSM_ACC_SUM); MNT4-753 (L = 27):
-    8 multiplications + 2 squarings."""
-    if L <= 13:
-        return 6 * imad_slots_per_mult(L) + 2 * imad_slots_per_sqr(L) + imad_slots_per_sum(L)
-    return 8 * imad_slots_per_mult(L) + 2 * imad_slots_per_sqr(L)
+    """PACC (Alg. 4) as implemented: 6 multiplications + 2 squarings + one fmul_sum
+    (Y' = R*D - Y*PPP with one reduction, ec.cuh MSM_ACC_SUM)."""
+    return 6 * imad_slots_per_mult(L) + 2 * imad_slots_per_sqr(L) + imad_slots_per_sum(L)
 
 
 def peaks():
@@ -572,9 +569,8 @@ def main():
                      "frac_pipe": achieved_slots / peak_imad,
                      "frac_pipe_basis": f"IMAD-pipe slots of the radix-2^{W} instruction stream run: {pacc} PACC x "
                                         f"{imad_slots_per_pacc(L)} slots ("
-                                        + (f"6 mul x {imad_slots_per_mult(L)} + 2 sqr x {imad_slots_per_sqr(L)} + 1 fmul_sum x "
-                                           f"{imad_slots_per_sum(L)}" if L <= 13 else
-                                           f"8 mul x {imad_slots_per_mult(L)} + 2 sqr x {imad_slots_per_sqr(L)}")
+                                        + f"6 mul x {imad_slots_per_mult(L)} + 2 sqr x {imad_slots_per_sqr(L)} + 1 fmul_sum x "
+                                          f"{imad_slots_per_sum(L)}"
                                         + "), IMAD.WIDE = 2 slots (measured)",
                      "field_mults_per_s": pacc * 10 / (acc_avg_ms / 1e3)},
         "clocks": clocks,

@@ -1181,14 +1181,14 @@ __global__ void __launch_bounds__(FIX_THREADS) k_fixup_long(uint32_t* __restrict
 //   descending running sum gives run = sum B_b and tri = sum (b - lo + 1) B_b;
 //   the segment's contribution is tri + (lo - 1) * run  (small-scalar double-and-add).
 // R = k * A by double-and-add over `bits` bits (warp-uniform trip count and call sequence)
-template <class C>
+template <class C, bool LAT = false>
 DEVI void xyzz_mul_small(Xyzz<C>& R, const Xyzz<C>& A, uint32_t k, int bits) {
   xyzz_set_zero<C>(R);
   Xyzz<C> Z;
   for (int b = bits - 1; b >= 0; b--) {
-    xyzz_dbl_ni<C>(R, R);
+    xyzz_dbl_sel_ni<C, LAT>(R, R);
     xyzz_select<C>(Z, A, (k >> b) & 1u);
-    xyzz_add_ni<C>(R, R, Z);
+    xyzz_add_sel_ni<C, LAT>(R, R, Z);
   }
 }
 
@@ -1198,7 +1198,9 @@ DEVI void xyzz_mul_small(Xyzz<C>& R, const Xyzz<C>& A, uint32_t k, int bits) {
 //   run = sum_q B_q,   tri = sum_q (q - lo) B_q          (2 PADD per bucket)
 // and the segment's share of W_j = sum_q (alpha q + beta) B_q is
 //   alpha*tri + (alpha*lo + beta)*run.
-template <class C>
+// LAT: latency-mode products — chosen when the segments fill less than half a wave (small
+// n: a few warps walk the serial chains; ops_impl.cuh)
+template <class C, bool LAT = false>
 __global__ void __launch_bounds__(SEG_NT, MSM_SEG_SYNC ? 1 : MSM_SEG_MINB) k_bucket_segments(const uint32_t* __restrict__ buckets, const uint32_t* __restrict__ goff,
                                                          int nwin, uint32_t NB, uint32_t seg, uint32_t nseg,
                                                          uint32_t alpha, uint32_t beta,
@@ -1221,16 +1223,16 @@ __global__ void __launch_bounds__(SEG_NT, MSM_SEG_SYNC ? 1 : MSM_SEG_MINB) k_buc
     const bool ne = live && b < NB && __ldg(goff + f + 1) != __ldg(goff + f);
     if (ne) load_xyzz<C>(B, buckets + f * XW);
     else xyzz_set_zero<C>(B);
-    xyzz_add_hot<C>(run, run, B);
-    if (q > 0) xyzz_add_hot<C>(tri, tri, run);  // warp-uniform: q is the same in every lane
+    xyzz_add_hot<C, LAT>(run, run, B);
+    if (q > 0) xyzz_add_hot<C, LAT>(tri, tri, run);  // warp-uniform: q is the same in every lane
   }
   if (alpha > 1) {  // warp-uniform
-    xyzz_mul_small<C>(B, tri, alpha, 32 - __clz(alpha));
+    xyzz_mul_small<C, LAT>(B, tri, alpha, 32 - __clz(alpha));
     tri = B;
   }
   const uint32_t kmax = alpha * (NB - 1) + beta;
-  xyzz_mul_small<C>(B, run, alpha * lo + beta, 32 - __clz(kmax | 1u));
-  xyzz_add_ni<C>(tri, tri, B);
+  xyzz_mul_small<C, LAT>(B, run, alpha * lo + beta, 32 - __clz(kmax | 1u));
+  xyzz_add_sel_ni<C, LAT>(tri, tri, B);
   if (live) store_xyzz<C>(out + (size_t)gid * XW, tri);
 }
 

@@ -136,7 +136,7 @@ struct Ops final : CurveOps {
     s.acc_threads = (uint32_t)std::max<size_t>(1, cdiv(Mmax, s.slice));
     // bucket-reduce segments
     int bps2 = 0;
-    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps2, k_bucket_segments<C>, SEG_NT, 0));
+    CK(cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps2, k_bucket_segments<C, false>, SEG_NT, 0));
     bps2 *= SEG_NT / 128;  // in units of 128 threads below
     if (bps2 < 1) bps2 = 1;
     const size_t resident2 = (size_t)sms * bps2 * 128;
@@ -145,6 +145,9 @@ struct Ops final : CurveOps {
     uint32_t seg = o.seg > 0 ? (uint32_t)o.seg : (uint32_t)std::max<size_t>(4, cdiv((size_t)s.nset * nb, resident2));
     s.seg = seg;
     s.nseg = (uint32_t)cdiv(nb, seg);
+    // latency-mode products (k_bucket_segments<C, true>): measured slower even below half a
+    // wave (C1 reduce 0.253 -> 0.269 ms, C2 1.073 -> 1.126 ms), so off; kept as an A/B
+    s.seg_lat = 0;
     if (!pre) free_table(s);
     else if (!s.table || s.table_c != c) {
       free_table(s);
@@ -344,8 +347,12 @@ struct Ops final : CurveOps {
     if (timed) CK(cudaEventRecord(s.ev[EV_FIX], st));
     // a5: bucket reduce
     const uint32_t total = (uint32_t)s.nset * s.nseg;
-    k_bucket_segments<C><<<(unsigned)cdiv(total, SEG_NT), SEG_NT, 0, st>>>(s.buckets, s.goff, s.nset, s.NB, s.seg, s.nseg,
-                                                                      (uint32_t)s.split_G, (uint32_t)s.split_g, s.segA);
+    if (s.seg_lat)
+      k_bucket_segments<C, true><<<(unsigned)cdiv(total, SEG_NT), SEG_NT, 0, st>>>(
+          s.buckets, s.goff, s.nset, s.NB, s.seg, s.nseg, (uint32_t)s.split_G, (uint32_t)s.split_g, s.segA);
+    else
+      k_bucket_segments<C, false><<<(unsigned)cdiv(total, SEG_NT), SEG_NT, 0, st>>>(
+          s.buckets, s.goff, s.nset, s.NB, s.seg, s.nseg, (uint32_t)s.split_G, (uint32_t)s.split_g, s.segA);
     launches++;
     uint32_t nin = s.nseg;
     uint32_t* src = s.segA;

@@ -58,6 +58,7 @@ struct Shard {
   size_t F = 0;        // flat buckets = nset * NB
   uint32_t acc_threads = 0, slice = 0;
   uint32_t seg = 0, nseg = 0;
+  int seg_lat = 0;     // bucket reduce with latency-mode products (small n)
   size_t ntiles = 0;
   // binned sort geometry (a3): flat bins fb = j*nbin + (b >> shift), FB = nwin*nbin
   int sort_mode = 0, shift = 0;  // effective a3 variant (1, 2 or 3)

@@ -185,12 +185,13 @@ def test_bench_gpus2_self_launch():
     """`python bench.py --gpus 2` without torchrun: bench.py re-launches itself with two
     ranks (shared-device mode when the box has one GPU) and rank 0 prints one JSON line
     whose closed-form check passes."""
-    cmd = [sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--log2n", "16", "--steps", "2",
-           "--warmup", "3", "--no-cpu-baseline", "--no-e2e"]
-    r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=ROOT)
-    assert r.returncode == 0, r.stderr[-3000:]
-    lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
-    assert len(lines) == 1, r.stdout
-    line = json.loads(lines[0])
-    assert line["n_gpus"] == 2
-    assert line["check"]["closed_form_match"] is True
+    for split in ("auto", "buckets"):  # auto = point shards in shared-device mode; buckets = f1 (PAPER.md:223)
+        cmd = [sys.executable, os.path.join(ROOT, "bench.py"), "--gpus", "2", "--log2n", "16", "--steps", "2",
+               "--warmup", "3", "--no-cpu-baseline", "--no-e2e", "--split", split]
+        r = subprocess.run(cmd, capture_output=True, text=True, timeout=600, cwd=ROOT)
+        assert r.returncode == 0, r.stderr[-3000:]
+        lines = [l for l in r.stdout.splitlines() if l.startswith("{")]
+        assert len(lines) == 1, r.stdout
+        line = json.loads(lines[0])
+        assert line["n_gpus"] == 2
+        assert line["check"]["closed_form_match"] is True, split

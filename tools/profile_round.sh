@@ -4,9 +4,9 @@
 #   dominant kernels.  Output under gpurun_out/prof/.
 cd "$(dirname "$0")/.."
 o=${OUT:-gpurun_out/prof}; mkdir -p $o
-B="python bench.py --steps 1 --warmup 3 --no-e2e --no-cpu-baseline ${BENCH_ARGS}"
+B="python bench.py --steps 1 --warmup 3 --no-e2e --no-cpu-baseline --no-check ${BENCH_ARGS}"
 [ -z "$NOLAUNCH" ] && timeout 900 ncu --metrics gpu__time_duration.sum --clock-control none -c 500 --csv --log-file $o/launches.csv \
-  python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu-baseline > $o/launches.log 2>&1
+  python bench.py --steps 2 --warmup 3 --no-e2e --no-cpu-baseline --no-check > $o/launches.log 2>&1
 for k in ${KERNELS:-k_accumulate k_bucket_segments k_s3_scatter}; do
   timeout 900 ncu --set full --clock-control none --import-source on -k regex:$k -s 1 -c 1 -o $o/$k -f $B > $o/$k.log 2>&1
   ncu -i $o/$k.ncu-rep --page raw --csv > $o/${k}_raw.csv 2>/dev/null
