@@ -310,8 +310,9 @@ def main():
     ap.add_argument("--window-bits", type=int, default=0)
     ap.add_argument("--precompute", type=int, default=2, choices=[0, 1, 2],
                     help="f3 window table (PAPER.md:147): 0 off, 1 on, 2 auto (library default)")
-    ap.add_argument("--sort", type=int, default=0, choices=[0, 1, 2, 3],
-                    help="a3 variant (MSM_OPT_SORT): 0 auto, 1 direct global atomics (ablation), 2 binned, 3 staged")
+    ap.add_argument("--sort", type=int, default=0, choices=[0, 1, 2, 3, 4],
+                    help="a3 variant (MSM_OPT_SORT): 0 auto, 1 direct global atomics (ablation), 2 binned, "
+                         "3 three-level staged, 4 two-pass cluster")
     ap.add_argument("--split", default="auto", choices=["auto", "points", "buckets"],
                     help="N > 1 decomposition: point shards, or the paper's bucket split (PAPER.md:223); "
                          "auto = buckets for N > 1")

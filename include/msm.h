@@ -78,7 +78,9 @@ enum {
   MSM_OPT_SEG_LEN = 3,        /* buckets per bucket-reduce segment; 0 = automatic          */
   MSM_OPT_SORT = 4,           /* a3 variant: 0 = auto (default: 3 for >= 2^21 entries, else 2),
                                  1 = direct global atomics (ablation), 2 = two-level binned,
-                                 3 = three-level staged (coalesced runs); get returns 1..3   */
+                                 3 = three-level staged (coalesced runs), 4 = two-pass
+                                 thread-block-cluster sort (ablation: half the HBM traffic of
+                                 3, slower on B200); get returns 1..4          */
   MSM_OPT_PRECOMPUTE = 5,     /* f3 window table 2^(jc) P_i: 0 off, 1 on,
                                  2 auto (default: on when the table fits in device memory).
                                  With it all windows share one bucket set; building the table

@@ -674,7 +674,7 @@ int msm_set_option(msm_context* ctx, int key, long value) {
       ctx->opt.seg = (int)value;
       break;
     case MSM_OPT_SORT:
-      if (value < 0 || value > 3) return MSM_ERR_ARG;
+      if (value < 0 || value > 4) return MSM_ERR_ARG;
       ctx->opt.sort = (int)value;
       break;
     case MSM_OPT_PRECOMPUTE:

@@ -10,6 +10,8 @@
 //   sorted   [M] u32          point index | sign << 31, grouped by flat bucket
 //   buckets  [F] Xyzz         bucket sums B_{j,b} (valid where the bucket is non-empty)
 #pragma once
+#include <cooperative_groups.h>
+
 #include "ec.cuh"
 
 namespace msmk {
@@ -555,6 +557,7 @@ __global__ void __launch_bounds__(BIN_THREADS) k_bin_scatter(const uint32_t* __r
 // scan helpers above.
 
 #include "sort3.cuh"
+#include "sort4.cuh"
 
 
 // ---------------------------------------------------------------------------------------

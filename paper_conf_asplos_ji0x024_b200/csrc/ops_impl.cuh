@@ -44,6 +44,7 @@ struct Ops final : CurveOps {
     dfree(s.s3Count); dfree(s.s3Off); dfree(s.s3Cursor); dfree(s.s3Sub);
     dfree(s.s3SubCount); dfree(s.s3SubCursor); dfree(s.s3Tiles);
     dfree(s.s3k1); dfree(s.s3v1); dfree(s.s3k2); dfree(s.s3v2);
+    dfree(s.s4Count); dfree(s.s4Off); dfree(s.s4Cursor); dfree(s.s4k); dfree(s.s4v);
     dfree(s.c4); dfree(s.goff4); dfree(s.cursor4); dfree(s.out4); dfree(s.baff_scratch);
     s.baff = 0;
   }
@@ -103,6 +104,17 @@ struct Ops final : CurveOps {
     // sort below ~2^21 entries (fewer launches)
     const size_t Mmax0 = s.n * (size_t)s.nwin;
     s.sort_mode = o.sort ? o.sort : (Mmax0 >= ((size_t)1 << 21) ? 3 : 2);
+    if (s.sort_mode == 4) {
+      // bins of 2^b2 flat buckets holding ~85 % of one cluster round (S4_CL * S4_CAP entries)
+      // on average; <= S4_MAXBIN bins, b2 in [3, 12] (else the three-level sort)
+      const double per_bucket = (double)std::max<size_t>(Mmax0 / (size_t)o.split_G, 1) / (double)std::max<size_t>(s.F, 1);
+      int b2 = (int)std::floor(std::log2(0.85 * S4_CL * S4_CAP / std::max(per_bucket, 1e-9)));
+      b2 = std::max(3, std::min(b2, 12));
+      while (b2 < 12 && ((s.F - 1) >> b2) + 1 > (size_t)S4_MAXBIN) b2++;
+      s.s4_b2 = b2;
+      s.s4_NC1 = (uint32_t)(((s.F - 1) >> b2) + 1);
+      if (s.s4_NC1 > (uint32_t)S4_MAXBIN) s.sort_mode = 3;
+    }
     s.shift = 0;
     while (s.shift < 13 && (size_t)s.nset * (((size_t)(s.NB - 1) >> s.shift) + 1) > 13000) s.shift++;
     s.nbin = (uint32_t)(((size_t)(s.NB - 1) >> s.shift) + 1);
@@ -210,6 +222,18 @@ struct Ops final : CurveOps {
       CK(cudaFuncSetAttribute(k_s3_part2, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * S3_TILE * 4));
       CK(cudaFuncSetAttribute(k_s3_part3, cudaFuncAttributeMaxDynamicSharedMemorySize, (S3_CAP + S3_MAXFINE) * 4));
     }
+    if (s.sort_mode == 4) {
+      const size_t NC1 = s.s4_NC1;
+      dalloc(&s.s4Count, NC1);
+      dalloc(&s.s4Off, NC1 + 1);
+      dalloc(&s.s4Cursor, NC1);
+      dalloc(&s.s4k, Mmax);
+      dalloc(&s.s4v, Mmax);
+      CK(cudaFuncSetAttribute(k_s4_count<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, (int)(NC1 * 4)));
+      CK(cudaFuncSetAttribute(k_s4_part1<C>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+                              (int)(12 * NC1 + 14 * (size_t)s4_t1((uint32_t)NC1))));
+      CK(cudaFuncSetAttribute(k_s4_part2, cudaFuncAttributeMaxDynamicSharedMemorySize, 3 * S4_MAXNBK * 4 + S4_CAP * 6));
+    }
     if (s.sort_mode == 2) {
       dalloc(&s.binCount, s.FB);
       dalloc(&s.binOff, s.FB + 1);
@@ -228,7 +252,32 @@ struct Ops final : CurveOps {
     const uint32_t* pts = s.pre ? s.table : s.pts;
     if (timed) CK(cudaEventRecord(s.ev[EV_H2D], st));
     // a2 + a3: digits, histogram, scan, scatter
-    if (s.sort_mode == 3) {
+    if (s.sort_mode == 4) {
+      const uint32_t NC1 = s.s4_NC1;
+      const int b2 = s.s4_b2;
+      CK(cudaMemsetAsync(s.s4Count, 0, NC1 * sizeof(uint32_t), st));
+      if (n) {
+        k_s4_count<C><<<(unsigned)cdiv(n, 512 * 16), 512, NC1 * 4, st>>>(scal, n, s.c_arg, s.nwin, ws, b2, NC1, s.s4Count,
+                                                                          s.err);
+        launches++;
+      }
+      const size_t nt = cdiv(NC1, SCAN_TILE);
+      k_scan_reduce<<<(unsigned)nt, SCAN_THREADS, 0, st>>>(s.s4Count, NC1, s.tiles);
+      k_scan_tiles<<<1, 1024, 0, st>>>(s.tiles, nt, s.s4Off + NC1);
+      k_scan_apply<<<(unsigned)nt, SCAN_THREADS, 0, st>>>(s.s4Count, NC1, s.tiles, s.s4Off, s.s4Cursor);
+      launches += 3;
+      if (n) {
+        const uint32_t tp = std::max<uint32_t>(1, s4_t1(NC1) / (uint32_t)s.nwin);
+        const size_t ctas = cdiv(cdiv(n, tp), S4_CL) * S4_CL;
+        k_s4_part1<C><<<(unsigned)ctas, S4_THREADS, 12 * NC1 + 14 * s4_t1(NC1), st>>>(
+            scal, n, s.c_arg, s.nwin, ws, istride, b2, NC1, tp, s.s4Cursor, s.s4k, s.s4v);
+        launches++;
+      }
+      CK(cudaMemcpyAsync(s.goff + s.F, s.s4Off + NC1, 4, cudaMemcpyDeviceToDevice, st));
+      k_s4_part2<<<(unsigned)(NC1 * S4_CL), S4_THREADS2, 3 * (4u << b2) + S4_CAP * 6, st>>>(s.s4Off, b2, (uint32_t)s.F,
+                                                                                         s.s4k, s.s4v, s.goff, s.sorted);
+      launches++;
+    } else if (s.sort_mode == 3) {
       const uint32_t NC1 = 1u << s.s3_b1, NC2 = 1u << s.s3_b2;
       const int sh1 = s.s3_b2 + s.s3_b3;
       CK(cudaMemsetAsync(s.s3Count, 0, NC1 * sizeof(uint32_t), st));

@@ -61,7 +61,7 @@ struct Shard {
   int seg_lat = 0;     // bucket reduce with latency-mode products (small n)
   size_t ntiles = 0;
   // binned sort geometry (a3): flat bins fb = j*nbin + (b >> shift), FB = nwin*nbin
-  int sort_mode = 0, shift = 0;  // effective a3 variant (1, 2 or 3)
+  int sort_mode = 0, shift = 0;  // effective a3 variant (1, 2, 3 or 4)
   uint32_t nbin = 0, FB = 0;
   size_t ntiles_bin = 0;
   // device buffers
@@ -80,6 +80,11 @@ struct Shard {
   uint32_t *s3Count = nullptr, *s3Off = nullptr, *s3Cursor = nullptr, *s3Sub = nullptr,
            *s3k1 = nullptr, *s3v1 = nullptr, *s3k2 = nullptr, *s3v2 = nullptr, *s3SubCount = nullptr,
            *s3SubCursor = nullptr, *s3Tiles = nullptr;
+  // two-pass cluster sort (sort4.cuh): bins of 2^s4_b2 flat buckets
+  int s4_b2 = 0;
+  uint32_t s4_NC1 = 0;
+  uint32_t *s4Count = nullptr, *s4Off = nullptr, *s4Cursor = nullptr, *s4v = nullptr;
+  uint16_t* s4k = nullptr;
   uint32_t* host_err = nullptr;  // pinned
   // f3 precomputation: table[j][i] = 2^(j c) P_i, affine device form,
   // [nwin][n][PW] words; built for window size table_c, kept across runs.
@@ -96,7 +101,7 @@ struct Shard {
 struct Options {
   int c = 0, threads = 0, seg = 0;
   int sort = 0;  // a3 variant: 0 auto, 1 direct global atomics (ablation), 2 two-level binned,
-                 // 3 three-level staged (sort3.cuh)
+                 // 3 three-level staged (sort3.cuh), 4 two-pass cluster (sort4.cuh)
   int pre = 2;   // f3 precomputation: 0 off, 1 on, 2 auto (on when the table fits in memory)
   int split_G = 1, split_g = 0;  // f1: this context sums only buckets |d| = G*q + g
   int acc_mode = 2;  // a4: 0 PACC only, 1 batch-affine front end + PACC (ablation), 2 auto (= 0, measured faster)

@@ -174,11 +174,12 @@ def test_device_resident_inputs(lib):
 
 
 @pytest.mark.parametrize("name", ["bn254", "bls12_381"])
-@pytest.mark.parametrize("sort", [1, 2, 3])
+@pytest.mark.parametrize("sort", [1, 2, 3, 4])
 @pytest.mark.parametrize("cbits", [4, 9, 13, 16])
 def test_sort_variants(lib, name, sort, cbits):
-    """a3 variants -- direct atomics (ablation), two-level binned, three-level staged -- all
-    give the oracle's result and the oracle's bucket sums, for bin shifts 0..> 0."""
+    """a3 variants -- direct atomics (ablation), two-level binned, three-level staged,
+    two-pass cluster -- all give the oracle's result and the oracle's bucket sums, for bin
+    shifts 0..> 0."""
     c = CURVES[name]
     n = 700
     Ps, es, _, _ = progression(name, n, 28)
@@ -207,7 +208,7 @@ def test_large_c_binned_sort(lib):
     Ps, es, _, _ = progression(name, n, 29)
     ks = synth.words_to_ints(synth.scalars(c.r, n, 41))
     ctx = lib.Context(name, points_to_words(list(Ps), name), n=n)
-    for sort in (2, 3):
+    for sort in (2, 3, 4):
         ctx.set_option(lib.OPT_SORT, sort)
         for pre in (0, 1):
             ctx.set_option(lib.OPT_PRECOMPUTE, pre)
@@ -217,10 +218,12 @@ def test_large_c_binned_sort(lib):
     ctx.close()
 
 
+@pytest.mark.parametrize("sort", [3, 4])
 @pytest.mark.parametrize("kind", ["ones", "skewed", "uniform"])
-def test_staged_sort_oversized_subbins(lib, kind):
-    """Three-level staged sort with > S3_CAP entries in one sub-bin (skewed scalars take
-    the global-scatter fallback of k_s3_part3) and on uniform scalars at several c."""
+def test_staged_sort_oversized_subbins(lib, kind, sort):
+    """Staged sorts on skewed scalars: three-level with > S3_CAP entries in one sub-bin (the
+    global-scatter fallback of k_s3_part3), two-pass cluster with bins of a few buckets;
+    and on uniform scalars at several c."""
     name = "bn254"
     c = CURVES[name]
     n = 20000
@@ -229,13 +232,13 @@ def test_staged_sort_oversized_subbins(lib, kind):
           else synth.words_to_ints(synth.pattern_scalars(c.r, n, 7, kind)))
     want = closed(name, ks, es)
     ctx = lib.Context(name, points_to_words(list(Ps), name), n=n)
-    ctx.set_option(lib.OPT_SORT, 3)
+    ctx.set_option(lib.OPT_SORT, sort)
     sw = synth.ints_to_words(ks, 8)
     for pre in (0, 1):
         ctx.set_option(lib.OPT_PRECOMPUTE, pre)
         for cbits in (5, 11, 16):
             ctx.set_option(lib.OPT_WINDOW_BITS, cbits)
-            assert ctx.get_option(lib.OPT_SORT) == 3
+            assert ctx.get_option(lib.OPT_SORT) == sort
             assert ctx.run(sw) == want, (pre, cbits)
     ctx.close()
 

@@ -195,3 +195,29 @@ def test_bench_gpus2_self_launch():
         line = json.loads(lines[0])
         assert line["n_gpus"] == 2
         assert line["check"]["closed_form_match"] is True, split
+
+
+@pytest.mark.parametrize("kind,cbits,pre", [("equal", 13, 1), ("skewed", 16, 1), ("uniform", 8, 1),
+                                            ("uniform", 16, 1), ("uniform", 12, 0)])
+def test_cluster_sort_heavy_bins(lib, kind, cbits, pre):
+    """Two-pass cluster sort (sort4.cuh) at n = 2^18 where bins exceed one cluster round
+    (S4_CL * S4_CAP = 196 608 entries): equal / skewed scalars put every entry in a few
+    buckets, c = 8 makes bins of 8 buckets holding ~2^20 entries each; the histogram sweep
+    and the rounds with running offsets must reproduce the closed form bit-exactly."""
+    name = "bls12_381"
+    c = CURVES[name]
+    n = 1 << 18
+    pts, es = gen_device_points(lib, name, n, 70)
+    ks_w = (synth.scalars_range(c.r, 0, n, 71) if kind == "uniform"
+            else synth.pattern_scalars(c.r, n, 72, kind))
+    ks = synth.words_to_ints(ks_w)
+    want = ec.to_output(ec.mul(sum(k * e for k, e in zip(ks, es)) % c.r, c.G, c))
+    ctx = lib.Context(name, pts, n=n)
+    try:
+        ctx.set_option(lib.OPT_SORT, 4)
+        ctx.set_option(lib.OPT_PRECOMPUTE, pre)
+        ctx.set_option(lib.OPT_WINDOW_BITS, cbits)
+        assert ctx.get_option(lib.OPT_SORT) == 4
+        assert ctx.run(ks_w) == want
+    finally:
+        ctx.close()
