@@ -464,6 +464,21 @@ def main():
                "h2d_bytes_per_step": n * S * 4, "d2h_bytes_per_step": 2 * L32 * 4,
                "timing": f"host wall clock around {nst} pipelined msm_submit/msm_wait calls (pinned host scalars, "
                          "each MSM's H2D overlaps the previous MSM's accumulation), per MSM"}
+        # single-call latency (one msm_run per MSM, pinned host scalars, H2D inside): the
+        # library default uploads the scalars in growing chunks, each sorted and accumulated
+        # while the next one uploads (MSM_OPT_H2D_CHUNKS); one copy before the MSM for contrast
+        single = {}
+        for K, key in ((0, "chunked"), (1, "one_copy")):
+            ctx.set_option(msm.OPT_H2D_CHUNKS, K)
+            ctx.run_words(ks_np)
+            ts = []
+            for _ in range(3):
+                s0 = time.perf_counter()
+                ctx.run_words(ks_np)
+                ts.append((time.perf_counter() - s0) * 1e3)
+            single[key] = {"ms": sorted(ts)[1], "chunks": int(ctx.get_option(msm.OPT_H2D_CHUNKS))}
+        ctx.set_option(msm.OPT_H2D_CHUNKS, 0)
+        e2e["single_call"] = dict(single, timing="host wall clock around msm_run (median of 3)")
     elif not args.no_e2e:
         for _ in range(1):
             step(ks_pinned)

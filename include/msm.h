@@ -103,6 +103,15 @@ enum {
                                  per-batch inversion made it 1.8x slower; mode 1
                                  exists for BN254 and BLS12-377/381 as an ablation);
                                  get returns the mode in use (0/1)                           */
+  MSM_OPT_H2D_CHUNKS = 9,     /* host scalars in msm_run / msm_run_partial: copy them in K
+                                 chunks of growing size (n/4^(K-1), 3n/4^(K-1), 12n/4^(K-1),
+                                 ...) on a copy stream, each sorted and accumulated INTO the
+                                 bucket set while the next one uploads ("can be
+                                 efficiently pipelined"); 0 = auto (default: K = 3 for
+                                 n >= 2^20 per shard where supported: BN254, BLS12-377/381 with
+                                 the staged or cluster sort), 1 = one copy before the MSM,
+                                 2..8 = K.  Device scalars are never chunked.  Get returns the
+                                 K used by the last run on shard 0.  No reconfiguration.      */
   MSM_OPT_NWIN = 101,         /* (get only) number of windows floor(lambda/c) + 1           */
   MSM_OPT_NSETS = 103,        /* (get only) bucket sets: nwin, or 1 with the f3 table        */
   MSM_OPT_NONEMPTY = 102,     /* (get only) non-empty buckets of the last run on shard 0    */

@@ -42,6 +42,8 @@ struct msm_context {
   uint32_t* d_result[MSM_MAX_INFLIGHT] = {};
   uint32_t* h_result = nullptr;  // pinned [MSM_MAX_INFLIGHT][2*L32 + 1] (last word: error flags)
   long next_ticket = 0, next_wait = 0;
+  uint32_t* h_run = nullptr;     // pinned [2*L32 + 1]: msm_run's result and error word (one D2H)
+  bool stats_pending = false;    // msm_stats of the last run are read lazily (msm_get_stats)
 };
 
 namespace {
@@ -197,18 +199,107 @@ void destroy_shard(CurveOps* ops, Shard& s) {
   s.host_err = nullptr;
   for (auto& e : s.ev)
     if (e) { cudaEventDestroy(e); e = nullptr; }
+  for (auto& e : s.cev)
+    if (e) { cudaEventDestroy(e); e = nullptr; }
+  if (s.gexec) cudaGraphExecDestroy(s.gexec);
+  if (s.graph) cudaGraphDestroy(s.graph);
+  s.gexec = nullptr;
+  s.graph = nullptr;
+  if (s.cstream) cudaStreamSynchronize(s.cstream), cudaStreamDestroy(s.cstream);
+  s.cstream = nullptr;
   if (s.stream) cudaStreamDestroy(s.stream);
   s.stream = nullptr;
 }
 
 int apply_window_bits(msm_context* ctx) {
+  Options o = ctx->opt;
+  if (o.c == 0 && o.tuned_c > 0) o.c = o.tuned_c;
   for (auto& s : ctx->shards) {
     int c = 0, pre = 0;
-    plan_shard(ctx->opt, s, ctx->ops->lambda(), ctx->ops->PW(), ctx->ops->XW(), &c, &pre,
+    plan_shard(o, s, ctx->ops->lambda(), ctx->ops->PW(), ctx->ops->XW(), &c, &pre,
                ctx->ops->L32() > 12 ? 3.5 : 4.4);
-    ctx->ops->configure(ctx->opt, s, c, pre);
+    ctx->ops->configure(o, s, c, pre);
+    s.gen++;  // invalidates the captured graph
   }
   return MSM_OK;
+}
+
+// Small n (2^10 <= n <= 2^17, one shard, c automatic): the cost model is a throughput
+// model, but here the MSM is a chain of dependent EC operations whose length depends on c in
+// ways it does not capture (the top window's lambda mod c bits pile n extra entries into a
+// few buckets -> long carry runs; the reduce's weight multiplication grows with c).  A
+// sweep (profiles/r02/small_n_c_sweep.txt: BN254 2^10 best c = 6 at 0.54 ms vs the model's
+// c = 10 at 0.69 ms; 2^12 c = 5; 2^14 c = 16; BLS12-381 2^16 c = 8) is non-monotonic, so the
+// context measures instead: each candidate c runs twice on hashed scalars and the fastest
+// second run wins (FFTW-style planning; ~0.1 s at creation).  MSM_NO_AUTOTUNE=1 disables it.
+void autotune_c(msm_context* ctx) {
+  Shard& s = ctx->shards[0];
+  std::vector<int> cands = {5, 6, 7, 8, 10, 12, 14, 16};
+  if (std::find(cands.begin(), cands.end(), s.c) == cands.end()) cands.push_back(s.c);
+  ctx->ops->rand_scalars(s, s.scal, s.n, 0x5eed1234u);
+  float best = 1e30f;
+  int bc = s.c;
+  for (int c : cands) {
+    ctx->opt.tuned_c = c;
+    apply_window_bits(ctx);
+    float ms = 0;
+    for (int rep = 0; rep < 2; rep++) {
+      CK(cudaMemsetAsync(s.err, 0, 4, s.stream));
+      CK(cudaEventRecord(s.ev[EV_START], s.stream));
+      ctx->ops->enqueue_pipeline(s, s.scal, false);
+      ctx->ops->enqueue_finalize(s.partial, 1, s.result, s.stream);
+      CK(cudaEventRecord(s.ev[EV_END], s.stream));
+      CK(cudaEventSynchronize(s.ev[EV_END]));
+      CK(cudaEventElapsedTime(&ms, s.ev[EV_START], s.ev[EV_END]));
+    }
+    if (ms < best) { best = ms; bc = c; }
+  }
+  ctx->opt.tuned_c = bc;
+  apply_window_bits(ctx);
+}
+
+// Small MSMs are launch-bound (C1: ~25 kernels for ~0.1 ms of GPU work), so for shards of
+// <= 2^17 points with device scalars on the shard's own device, a2..a6 are captured into a
+// CUDA graph the second time the same scalar buffer is seen, and replayed after that.
+constexpr size_t GRAPH_MAX_N = (size_t)1 << 17;
+// A replayed graph has no per-stage events: the stage events are recorded after it (the
+// stats then show the whole a2..a6 time as sort_ms and 0 for the later stages), which also
+// keeps EV_SORT valid for msm_submit's copy-stream ordering.
+void graph_launch(Shard& s, bool timed) {
+  if (timed) CK(cudaEventRecord(s.ev[EV_H2D], s.stream));
+  CK(cudaGraphLaunch(s.gexec, s.stream));
+  if (timed)
+    for (int e : {EV_SORT, EV_BAFF, EV_ACC, EV_FIX, EV_RED, EV_COMB}) CK(cudaEventRecord(s.ev[e], s.stream));
+}
+int enqueue_graphed(msm_context* ctx, Shard& s, const uint32_t* sc, bool timed) {
+  const bool same = sc == s.last_scal;
+  s.last_scal = sc;
+  if (s.gexec && s.g_gen == s.gen && s.g_scal == sc) {
+    graph_launch(s, timed);
+    return s.g_launches;
+  }
+  if (!same) return ctx->ops->enqueue_pipeline(s, sc, timed);
+  if (s.gexec) cudaGraphExecDestroy(s.gexec);
+  if (s.graph) cudaGraphDestroy(s.graph);
+  s.gexec = nullptr;
+  s.graph = nullptr;
+  CK(cudaStreamBeginCapture(s.stream, cudaStreamCaptureModeThreadLocal));
+  int launched = 0;
+  try {
+    launched = ctx->ops->enqueue_pipeline(s, sc, false);  // no event nodes in the graph
+  } catch (...) {
+    cudaGraph_t g = nullptr;
+    cudaStreamEndCapture(s.stream, &g);
+    if (g) cudaGraphDestroy(g);
+    throw;
+  }
+  CK(cudaStreamEndCapture(s.stream, &s.graph));
+  CK(cudaGraphInstantiate(&s.gexec, s.graph, 0));
+  s.g_gen = s.gen;
+  s.g_scal = sc;
+  s.g_launches = launched;
+  graph_launch(s, timed);
+  return launched;
 }
 
 // scalar pointer for shard s: device-resident on the shard's device -> use directly,
@@ -226,6 +317,43 @@ const uint32_t* stage_scalars(msm_context* ctx, Shard& s, const uint32_t* scalar
     CK(cudaMemcpyAsync(s.scal, src, bytes, cudaMemcpyHostToDevice, s.stream));
   }
   return s.scal;
+}
+
+// Host scalars in K chunks (the bucket work "can be efficiently pipelined"
+// with the transfers): chunk k's H2D runs on the shard's copy stream while the compute
+// stream sorts and accumulates chunk k-1 into the bucket set.  Chunk sizes grow by 4x
+// (n/4^(K-1), 3n/4^(K-1), 12n/4^(K-1), ...): the GPU work of a chunk (~6 GB/s of scalars
+// at 2^26) outlasts the next chunk's copy (25-50 GB/s), so only the first, smallest copy
+// stays on the critical path.  Each later chunk costs one extra PACC per non-empty bucket
+// (INIT accumulation from the stored bucket).
+int h2d_chunks(msm_context* ctx, const Shard& s) {
+  const int want = ctx->opt.chunks;
+  if (want == 1 || s.n == 0 || !ctx->ops->can_chunk(s)) return 1;
+  if (want == 0) return s.n >= ((size_t)1 << 20) ? 3 : 1;
+  return std::min(want, 8);
+}
+
+int run_chunked(msm_context* ctx, Shard& s, const uint32_t* host_src, int K, bool timed) {
+  const size_t S = ctx->ops->S();
+  if (!s.cstream) CK(cudaStreamCreateWithFlags(&s.cstream, cudaStreamNonBlocking));
+  for (int k = 0; k < K; k++)
+    if (!s.cev[k]) CK(cudaEventCreateWithFlags(&s.cev[k], cudaEventDisableTiming));
+  // the copy stream must not overwrite s.scal while an earlier MSM on s.stream reads it
+  CK(cudaEventRecord(s.cev[0], s.stream));
+  CK(cudaStreamWaitEvent(s.cstream, s.cev[0], 0));
+  const double T = std::pow(4.0, K - 1);
+  int launched = 0;
+  size_t lo = 0;
+  for (int k = 0; k < K; k++) {
+    const size_t hi = k == K - 1 ? s.n : std::min(s.n, (size_t)std::llround((double)s.n * std::pow(4.0, k) / T));
+    if (hi < lo) continue;
+    CK(cudaMemcpyAsync(s.scal + lo * S, host_src + lo * S, (hi - lo) * S * 4, cudaMemcpyHostToDevice, s.cstream));
+    CK(cudaEventRecord(s.cev[k], s.cstream));
+    CK(cudaStreamWaitEvent(s.stream, s.cev[k], 0));
+    launched += ctx->ops->enqueue_chunk(s, s.scal + lo * S, hi - lo, lo, k == 0, k == K - 1, timed && k == K - 1);
+    lo = hi;
+  }
+  return launched;
 }
 
 int check_errors(msm_context* ctx) {
@@ -258,9 +386,20 @@ int run_all(msm_context* ctx, const uint32_t* scalars, bool gather_to_dev0) {
       if (is_dev) order_after_legacy(src_dev, s.dev, s.stream);
       if (timed) CK(cudaEventRecord(s.ev[EV_START], s.stream));
       CK(cudaMemsetAsync(s.err, 0, 4, s.stream));
-      const uint32_t* sc = stage_scalars(ctx, s, scalars, is_dev, src_dev);
-      NvtxRange nr("enqueue a2..a6 (shard)");
-      launched[g] = ctx->ops->enqueue_pipeline(s, sc, timed);
+      const int K = is_dev ? 1 : h2d_chunks(ctx, s);
+      s.chunks_used = K;
+      if (K > 1) {
+        NvtxRange nr("chunked H2D + a2..a6 (shard)");
+        launched[g] = run_chunked(ctx, s, scalars + s.off * ctx->ops->S(), K, timed);
+      } else {
+        const uint32_t* sc = stage_scalars(ctx, s, scalars, is_dev, src_dev);
+        NvtxRange nr("enqueue a2..a6 (shard)");
+        static const bool no_graph = getenv("MSM_NO_GRAPH") != nullptr;  // A/B
+        if (!no_graph && is_dev && src_dev == s.dev && s.n <= GRAPH_MAX_N && sc != s.scal)
+          launched[g] = enqueue_graphed(ctx, s, sc, timed);
+        else
+          launched[g] = ctx->ops->enqueue_pipeline(s, sc, timed);
+      }
     } catch (const CudaError& e) {
       rc[g] = e.code;
     } catch (...) {
@@ -491,7 +630,11 @@ msm_context* msm_context_create_on(int curve, const uint32_t* points, size_t n, 
           }
         }
     }
-    return apply_window_bits(ctx);
+    const int e2 = apply_window_bits(ctx);
+    if (e2 != MSM_OK) return e2;
+    static const bool no_tune = getenv("MSM_NO_AUTOTUNE") != nullptr;
+    if (!no_tune && ngpus == 1 && n >= ((size_t)1 << 10) && n <= ((size_t)1 << 17)) autotune_c(ctx);
+    return MSM_OK;
   });
   if (rc != MSM_OK) {
     g_last_error = rc;
@@ -517,6 +660,7 @@ void msm_context_destroy(msm_context* ctx) {
     }
     cudaFreeHost(ctx->h_result);
   }
+  if (ctx->h_run) cudaFreeHost(ctx->h_run);
   for (auto& s : ctx->shards) destroy_shard(ctx->ops, s);
   delete ctx;
 }
@@ -531,10 +675,22 @@ int msm_run(msm_context* ctx, const uint32_t* scalars, uint32_t* result) {
     ctx->ops->enqueue_finalize(s0.partials, (int)ctx->shards.size(), s0.result, s0.stream);
     ctx->launches++;
     CK(cudaEventRecord(s0.ev[EV_END], s0.stream));
+    ctx->stats_pending = true;
+    const int L32 = ctx->ops->L32();
+    if (ctx->shards.size() == 1) {  // one round trip: result and error word together
+      if (!ctx->h_run) CK(cudaMallocHost((void**)&ctx->h_run, (2 * 24 + 1) * 4));
+      CK(cudaMemcpyAsync(ctx->h_run, s0.result, 2 * L32 * 4, cudaMemcpyDeviceToHost, s0.stream));
+      CK(cudaMemcpyAsync(ctx->h_run + 2 * L32, s0.err, 4, cudaMemcpyDeviceToHost, s0.stream));
+      CK(cudaStreamSynchronize(s0.stream));
+      const uint32_t e = ctx->h_run[2 * L32];
+      if (e & 4u) return MSM_ERR_SCALAR;
+      if (e & 3u) return MSM_ERR_POINT;
+      std::memcpy(result, ctx->h_run, 2 * L32 * 4);
+      return MSM_OK;
+    }
     const int e = check_errors(ctx);
-    collect_stats(ctx);
     if (e != MSM_OK) return e;
-    CK(cudaMemcpy(result, s0.result, 2 * ctx->ops->L32() * 4, cudaMemcpyDeviceToHost));
+    CK(cudaMemcpy(result, s0.result, 2 * L32 * 4, cudaMemcpyDeviceToHost));
     return MSM_OK;
   });
 }
@@ -548,7 +704,7 @@ int msm_run_partial(msm_context* ctx, const uint32_t* scalars, uint32_t* partial
     CK(cudaSetDevice(s0.dev));
     CK(cudaEventRecord(s0.ev[EV_END], s0.stream));
     const int e = check_errors(ctx);
-    collect_stats(ctx);
+    ctx->stats_pending = true;
     if (e != MSM_OK) return e;
     int pdev = -1;
     if (is_device_ptr(partial, &pdev)) {
@@ -614,7 +770,10 @@ int msm_wait(msm_context* ctx, long ticket, uint32_t* result) {
     CK(cudaSetDevice(s.dev));
     CK(cudaEventSynchronize(ctx->ev_done[q]));
     ctx->next_wait++;
-    if (ticket + 1 == ctx->next_ticket) collect_stats(ctx);
+    if (ticket + 1 == ctx->next_ticket) {
+      collect_stats(ctx);
+      ctx->stats_pending = false;
+    }
     const uint32_t* h = ctx->h_result + q * (2 * L32 + 1);
     const uint32_t e = h[2 * L32];
     if (e & 4u) return MSM_ERR_SCALAR;
@@ -695,6 +854,10 @@ int msm_set_option(msm_context* ctx, int key, long value) {
       if (value == 1 && !ctx->ops->has_baff()) return MSM_ERR_UNIMPLEMENTED;
       ctx->opt.acc_mode = (int)value;
       break;
+    case MSM_OPT_H2D_CHUNKS:
+      if (value < 0 || value > 8) return MSM_ERR_ARG;
+      ctx->opt.chunks = (int)value;
+      return MSM_OK;  // no reconfiguration
     default:
       return MSM_ERR_ARG;
   }
@@ -714,6 +877,7 @@ long msm_get_option(msm_context* ctx, int key) {
     case MSM_OPT_SPLIT_PARTS: return ctx->opt.split_G;
     case MSM_OPT_SPLIT_INDEX: return ctx->opt.split_g;
     case MSM_OPT_ACC_MODE: return ctx->shards[0].baff;
+    case MSM_OPT_H2D_CHUNKS: return ctx->shards[0].chunks_used;
     case MSM_OPT_DEVICE: return ctx->shards[0].dev;
     case MSM_OPT_NGPUS: return (long)ctx->shards.size();
     case MSM_OPT_NONEMPTY: {
@@ -727,6 +891,15 @@ long msm_get_option(msm_context* ctx, int key) {
 
 int msm_get_stats(const msm_context* ctx, msm_stats* out) {
   if (!ctx || !out) return MSM_ERR_ARG;
+  if (ctx->stats_pending) {  // read the events and counters of the last run now, not in msm_run
+    msm_context* c = const_cast<msm_context*>(ctx);
+    const int rc = guarded([&]() -> int {
+      collect_stats(c);
+      return MSM_OK;
+    });
+    if (rc != MSM_OK) return rc;
+    c->stats_pending = false;
+  }
   *out = ctx->stats;
   return MSM_OK;
 }

@@ -559,84 +559,157 @@ __device__ __noinline__ void finv(uint32_t* r, const uint32_t* a) {
   fcopy<C>(r, acc);
 }
 
-// r = a^-1 (Montgomery form in and out; a != 0 mod p) by the binary extended Euclidean
-// algorithm on canonical 32-bit words (PAPER.md is silent on inversion; R19).
-// Used by the single-thread final normalisation (a7), where Fermat's ~|p| serial
-// latency-mode products dominate (0.75 ms for BLS12-381); the binary GCD is ~2|p| cheap
-// shift/subtract steps.  Variable time: the MSM result is not secret.  Invariants (odd p):
-//   x1 * a == u (mod p),  x2 * a == v (mod p),  x1, x2 in [0, p),  gcd(u, v) = 1.
-// The word result is inv(aR) = a^-1 R^-1; two Montgomery products by R^2 give a^-1 R.
+// r = a^-1 (Montgomery form in and out; a != 0 mod p) by binary GCD on canonical 32-bit
+// words (PAPER.md is silent on inversion; R19), for the single-thread final
+// normalisation (a7), where Fermat's ~|p| serial latency-mode products dominate (0.75 ms
+// for BLS12-381).  Round 2: the batched form of Pornin ("Optimized binary GCD for modular
+// inversion", 2020): the binary-GCD step (a odd: if a < b swap (a,u),(b,v); a -= b,
+// u -= v; then a /= 2, u /= 2 mod p) runs 30 times on 62-bit approximations of a and b
+// (their low 30 bits, exact, and their top 32 bits), recording the steps as a 2x2 matrix
+// of signed factors (|f| + |g| <= 2^30); then (a, b) <- (f0 a + g0 b, f1 a + g1 b) / 2^30
+// (negated if an approximate comparison made one negative) and (u, v) likewise mod p.
+// ceil((2|p| - 1) / 30) batches suffice; invariants a == u*y, b == v*y (mod p), and b = 1,
+// v = y^-1 at the end.  Variable time: the MSM result is not secret.  Input words
+// y = canonical(aR) = aR mod p; output (aR)^-1, then two Montgomery products by R^2 give
+// a^-1 R.
+template <int N>
+DEVI uint32_t inv_words_bits(const uint32_t* w, int pos) {  // bits [pos, pos + 32) of w
+  const int q = pos >> 5, sh = pos & 31;
+  const uint32_t lo = q < N ? w[q] : 0u, hi = q + 1 < N ? w[q + 1] : 0u;
+  return sh ? (lo >> sh) | (hi << (32 - sh)) : lo;
+}
+// r = (f x + g y) / 2^30 (exact), |r| returned with neg = sign; N words
+template <int N>
+DEVI void inv_lin_shift(uint32_t* r, const uint32_t* x, const uint32_t* y, int64_t f, int64_t g, bool& neg) {
+  uint32_t t[N + 1];
+  int64_t c = 0;
+#pragma unroll
+  for (int i = 0; i < N; i++) {
+    const int64_t s = f * (int64_t)x[i] + g * (int64_t)y[i] + c;
+    t[i] = (uint32_t)s;
+    c = s >> 32;
+  }
+  t[N] = (uint32_t)c;
+  neg = c < 0;
+  if (neg) {  // two's complement over N + 1 words
+    uint32_t cy = 1;
+#pragma unroll
+    for (int i = 0; i <= N; i++) {
+      const uint64_t s2 = (uint64_t)(~t[i]) + cy;
+      t[i] = (uint32_t)s2;
+      cy = (uint32_t)(s2 >> 32);
+    }
+  }
+#pragma unroll
+  for (int i = 0; i < N; i++) r[i] = (t[i] >> 30) | (t[i + 1] << 2);
+}
+// r = (f x + g y) / 2^30 mod p, x, y in [0, p), r in [0, p); minv = -p^-1 mod 2^30
+template <int N>
+DEVI void inv_lin_mod(uint32_t* r, const uint32_t* x, const uint32_t* y, int64_t f, int64_t g,
+                      const uint32_t* p, uint32_t minv) {
+  uint32_t t[N + 1];
+  int64_t c = 0;
+#pragma unroll
+  for (int i = 0; i < N; i++) {
+    const int64_t s = f * (int64_t)x[i] + g * (int64_t)y[i] + c;
+    t[i] = (uint32_t)s;
+    c = s >> 32;
+  }
+  t[N] = (uint32_t)c;
+  const uint32_t q = (t[0] * minv) & 0x3fffffffu;  // t + q p == 0 mod 2^30
+  uint64_t cy = 0;
+#pragma unroll
+  for (int i = 0; i < N; i++) {
+    cy += (uint64_t)q * p[i] + t[i];
+    t[i] = (uint32_t)cy;
+    cy >>= 32;
+  }
+  t[N] += (uint32_t)cy;  // two's complement top word; the true value is in (-2^30 p, 2^31 p)
+  uint32_t w[N + 1];
+#pragma unroll
+  for (int i = 0; i < N; i++) w[i] = (t[i] >> 30) | (t[i + 1] << 2);
+  w[N] = (uint32_t)((int32_t)t[N] >> 30);  // r in (-p, 2p)
+  if ((int32_t)w[N] < 0) {  // += p
+    uint64_t s = 0;
+#pragma unroll
+    for (int i = 0; i < N; i++) { s += (uint64_t)w[i] + p[i]; w[i] = (uint32_t)s; s >>= 32; }
+    w[N] += (uint32_t)s;
+  } else {  // -= p if >= p
+    bool ge = w[N] != 0;
+    if (!ge) {
+      bool done = false;
+      ge = true;
+#pragma unroll
+      for (int i = N - 1; i >= 0; i--)
+        if (!done && w[i] != p[i]) { ge = w[i] > p[i]; done = true; }
+    }
+    if (ge) {
+      int64_t s = 0;
+#pragma unroll
+      for (int i = 0; i < N; i++) { s = (int64_t)w[i] - p[i] + (s >> 32); w[i] = (uint32_t)s; }
+    }
+  }
+#pragma unroll
+  for (int i = 0; i < N; i++) r[i] = w[i];
+}
+
 template <class C>
 __device__ __noinline__ void finv_bgcd(uint32_t* r, const uint32_t* a) {
   constexpr int N = C::L32;
-  uint32_t t[C::L], u[N], v[N], x1[N], x2[N], p[N];
+  uint32_t t[C::L], ua[N], ub[N], u[N], v[N], p[N];
   fcopy<C>(t, a);
   freduce<C>(t);
-  to_words32<C>(u, t);
+  to_words32<C>(ua, t);
+  uint32_t nz = 0;
 #pragma unroll
-  for (int i = 0; i < N; i++) { p[i] = C::P32c()[i]; v[i] = p[i]; x1[i] = 0; x2[i] = 0; }
-  x1[0] = 1;
-  {
-    uint32_t nz = 0;
-#pragma unroll
-    for (int i = 0; i < N; i++) nz |= u[i];
-    if (nz == 0) {  // a == 0 mod p has no inverse: return 0 rather than loop
-      fzero<C>(r);
-      return;
-    }
+  for (int i = 0; i < N; i++) { p[i] = C::P32c()[i]; ub[i] = p[i]; u[i] = i == 0; v[i] = 0; nz |= ua[i]; }
+  if (nz == 0) {  // a == 0 mod p has no inverse: return 0 rather than loop
+    fzero<C>(r);
+    return;
   }
-  auto is_one = [&](const uint32_t* w) {
-    uint32_t o = w[0] ^ 1u;
+  uint32_t pinv = p[0];  // p^-1 mod 2^32 by Newton (p odd: correct to 3 bits, doubling)
 #pragma unroll
-    for (int i = 1; i < N; i++) o |= w[i];
-    return o == 0;
-  };
-  // w >>= 1; x = x/2 mod p  (x + p when x is odd; the carry out of the top word is bit 32N)
-  auto halve = [&](uint32_t* w, uint32_t* x) {
-#pragma unroll
-    for (int i = 0; i < N - 1; i++) w[i] = __funnelshift_r(w[i], w[i + 1], 1);
-    w[N - 1] >>= 1;
-    uint32_t c = 0;
-    if (x[0] & 1u) {
-      u64 s = 0;
-#pragma unroll
-      for (int i = 0; i < N; i++) { s = (u64)x[i] + p[i] + (s >> 32); x[i] = (uint32_t)s; }
-      c = (uint32_t)(s >> 32);
+  for (int k = 0; k < 4; k++) pinv *= 2u - p[0] * pinv;
+  const uint32_t minv = (0u - pinv) & 0x3fffffffu;
+  const int pbits = 32 * N - __clz(p[N - 1]);
+  const int batches = (2 * pbits - 1 + 29) / 30;
+  for (int it = 0; it < batches; it++) {
+    int top = N - 1;
+    while (top > 0 && (ua[top] | ub[top]) == 0) top--;
+    const int len = 32 * top + 32 - __clz(ua[top] | ub[top]);
+    const int nb = len > 62 ? len : 62;
+    uint64_t A = (ua[0] & 0x3fffffffu) | ((uint64_t)inv_words_bits<N>(ua, nb - 32) << 30);
+    uint64_t B = (ub[0] & 0x3fffffffu) | ((uint64_t)inv_words_bits<N>(ub, nb - 32) << 30);
+    int64_t f0 = 1, g0 = 0, f1 = 0, g1 = 1;
+    for (int j = 0; j < 30; j++) {
+      if (A & 1u) {
+        if (A < B) {
+          const uint64_t T = A; A = B; B = T;
+          int64_t q = f0; f0 = f1; f1 = q;
+          q = g0; g0 = g1; g1 = q;
+        }
+        A -= B;
+        f0 -= f1;
+        g0 -= g1;
+      }
+      A >>= 1;
+      f1 *= 2;
+      g1 *= 2;
     }
+    uint32_t na[N], nb2[N];
+    bool neg_a, neg_b;
+    inv_lin_shift<N>(na, ua, ub, f0, g0, neg_a);
+    inv_lin_shift<N>(nb2, ua, ub, f1, g1, neg_b);
+    if (neg_a) { f0 = -f0; g0 = -g0; }
+    if (neg_b) { f1 = -f1; g1 = -g1; }
+    uint32_t nu[N], nv[N];
+    inv_lin_mod<N>(nu, u, v, f0, g0, p, minv);
+    inv_lin_mod<N>(nv, u, v, f1, g1, p, minv);
 #pragma unroll
-    for (int i = 0; i < N - 1; i++) x[i] = __funnelshift_r(x[i], x[i + 1], 1);
-    x[N - 1] = (x[N - 1] >> 1) | (c << 31);
-  };
-  // w -= z (w >= z);  x = x - y mod p
-  auto sub_step = [&](uint32_t* w, const uint32_t* z, uint32_t* x, const uint32_t* y) {
-    int64_t s = 0;
-#pragma unroll
-    for (int i = 0; i < N; i++) { s = (int64_t)w[i] - z[i] + (s >> 32); w[i] = (uint32_t)s; }
-    s = 0;
-#pragma unroll
-    for (int i = 0; i < N; i++) { s = (int64_t)x[i] - y[i] + (s >> 32); x[i] = (uint32_t)s; }
-    if (s < 0) {  // borrow: add p back
-      u64 q = 0;
-#pragma unroll
-      for (int i = 0; i < N; i++) { q = (u64)x[i] + p[i] + (q >> 32); x[i] = (uint32_t)q; }
-    }
-  };
-  auto geq = [&](const uint32_t* w, const uint32_t* z) {
-    bool ge = true, done = false;
-#pragma unroll
-    for (int i = N - 1; i >= 0; i--) {
-      if (!done && w[i] != z[i]) { ge = w[i] > z[i]; done = true; }
-    }
-    return ge;
-  };
-  while (!is_one(u) && !is_one(v)) {
-    while (!(u[0] & 1u)) halve(u, x1);
-    while (!(v[0] & 1u)) halve(v, x2);
-    if (geq(u, v)) sub_step(u, v, x1, x2);
-    else sub_step(v, u, x2, x1);
+    for (int i = 0; i < N; i++) { ua[i] = na[i]; ub[i] = nb2[i]; u[i] = nu[i]; v[i] = nv[i]; }
   }
   uint32_t w[C::L], r2[C::L];
-  from_words32<C>(w, is_one(u) ? x1 : x2);
+  from_words32<C>(w, v);  // b == 1: v = y^-1
 #pragma unroll
   for (int i = 0; i < C::L; i++) r2[i] = C::R2(i);
   fmul_lat<C>(w, w, r2);  // a^-1 R^-1 -> a^-1

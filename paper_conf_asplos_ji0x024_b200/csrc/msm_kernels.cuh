@@ -758,7 +758,11 @@ DEVI uint32_t entry_at(const uint32_t* __restrict__ sorted, uint32_t e) {
   else return __ldg(sorted + e);
 }
 
-template <class C, bool DIRECT = false>
+// INIT (chunked host scalars, engine.cu): the buckets already hold the sums of earlier
+// chunks, so a thread that owns a bucket's first entry starts from the stored bucket (O
+// if it was empty) and adds the entry by PACC instead of starting from the entry; the loop
+// then begins at the slice's first entry (every lane one more iteration, still uniform).
+template <class C, bool DIRECT = false, bool INIT = false>
 __global__ void __launch_bounds__(ACC_SYNC_NT, 1) k_accumulate_sync(const uint32_t* __restrict__ pts, const uint32_t* __restrict__ sorted,
                                                     const uint32_t* __restrict__ goff, uint32_t F,
                                                     uint32_t* __restrict__ buckets, uint32_t* __restrict__ carry_pts,
@@ -783,21 +787,28 @@ __global__ void __launch_bounds__(ACC_SYNC_NT, 1) k_accumulate_sync(const uint32
   // next point into registers one PACC ahead (L <= 13), or an L1 prefetch for MNT4-753
   // whose 255 registers leave no room for it
   constexpr bool REGPF = C::L <= 13;
+  // INIT: the first entry goes through the loop (q = 0) like every other one
+  constexpr uint32_t Q0 = INIT ? 0u : 1u;
   if (active) {
     f = find_bucket(goff, F, e0);
     end = __ldg(goff + f + 1);
     head = __ldg(goff + f) < e0;
-    ok = point_for_entry<C>(x, y, pts, entry_at<DIRECT>(sorted, e0));
-    acc_start<C>(acc, x, y, ok);
-    ent1 = e0 + 1 < e1 ? entry_at<DIRECT>(sorted, e0 + 1) : 0u;
-    ent2 = e0 + 2 < e1 ? entry_at<DIRECT>(sorted, e0 + 2) : 0u;
-    if constexpr (REGPF) {
-      if (e0 + 1 < e1) load_point<C>(nx, ny, pts, ent1 & ~SIGN_BIT);
+    if constexpr (INIT) {
+      if (head) xyzz_set_zero<C>(acc);
+      else load_xyzz<C>(acc, buckets + (size_t)f * XW);
     } else {
-      if (e0 + 1 < e1) prefetch_point<C>(pts, ent1);
+      ok = point_for_entry<C>(x, y, pts, entry_at<DIRECT>(sorted, e0));
+      acc_start<C>(acc, x, y, ok);
+    }
+    ent1 = e0 + Q0 < e1 ? entry_at<DIRECT>(sorted, e0 + Q0) : 0u;
+    ent2 = e0 + Q0 + 1 < e1 ? entry_at<DIRECT>(sorted, e0 + Q0 + 1) : 0u;
+    if constexpr (REGPF) {
+      if (e0 + Q0 < e1) load_point<C>(nx, ny, pts, ent1 & ~SIGN_BIT);
+    } else {
+      if (e0 + Q0 < e1) prefetch_point<C>(pts, ent1);
     }
   }
-  for (uint32_t q = 1; q < slice; q++) {
+  for (uint32_t q = Q0; q < slice; q++) {
     __syncthreads();
     const uint32_t e = e0 + q;
     if (!active || e >= e1) continue;
@@ -815,15 +826,30 @@ __global__ void __launch_bounds__(ACC_SYNC_NT, 1) k_accumulate_sync(const uint32
       if (e + 2 < e1) ent2 = entry_at<DIRECT>(sorted, e + 2);
       ok = point_for_entry<C>(x, y, pts, ent);
     }
-    if (e == end) {
-      if (head) { store_xyzz<C>(carry_pts + (size_t)t * XW, acc); my_carry = (int32_t)f; head = false; }
-      else store_xyzz<C>(buckets + (size_t)f * XW, acc);
-      do { f++; end = __ldg(goff + f + 1); } while (end <= e);
-      acc_start<C>(acc, x, y, ok);
-    } else if (ok) {
-      if (xyzz_acc_hot<C>(acc, x, y)) {
-        Xyzz<C> T = acc;
-        xyzz_dbl<C>(acc, T);
+    if constexpr (INIT) {
+      if (e == end) {
+        if (head) { store_xyzz<C>(carry_pts + (size_t)t * XW, acc); my_carry = (int32_t)f; head = false; }
+        else store_xyzz<C>(buckets + (size_t)f * XW, acc);
+        do { f++; end = __ldg(goff + f + 1); } while (end <= e);
+        load_xyzz<C>(acc, buckets + (size_t)f * XW);
+      }
+      if (ok) {
+        if (xyzz_acc_hot<C>(acc, x, y)) {
+          Xyzz<C> T = acc;
+          xyzz_dbl<C>(acc, T);
+        }
+      }
+    } else {
+      if (e == end) {
+        if (head) { store_xyzz<C>(carry_pts + (size_t)t * XW, acc); my_carry = (int32_t)f; head = false; }
+        else store_xyzz<C>(buckets + (size_t)f * XW, acc);
+        do { f++; end = __ldg(goff + f + 1); } while (end <= e);
+        acc_start<C>(acc, x, y, ok);
+      } else if (ok) {
+        if (xyzz_acc_hot<C>(acc, x, y)) {
+          Xyzz<C> T = acc;
+          xyzz_dbl<C>(acc, T);
+        }
       }
     }
   }
@@ -1223,7 +1249,8 @@ __global__ void __launch_bounds__(SEG_NT, MSM_SEG_SYNC ? 1 : MSM_SEG_MINB) k_buc
     if (MSM_SEG_SYNC) __syncthreads();  // lockstep: shared instruction fetch (see k_accumulate_sync)
     const uint32_t b = lo + q;
     const size_t f = (size_t)j * NB + b;
-    const bool ne = live && b < NB && __ldg(goff + f + 1) != __ldg(goff + f);
+    // goff == nullptr (chunked host scalars): every bucket was written (zeroed = O first)
+    const bool ne = live && b < NB && (goff == nullptr || __ldg(goff + f + 1) != __ldg(goff + f));
     if (ne) load_xyzz<C>(B, buckets + f * XW);
     else xyzz_set_zero<C>(B);
     xyzz_add_hot<C, LAT>(run, run, B);
@@ -1369,6 +1396,19 @@ __global__ void k_gen_bases(const uint32_t* __restrict__ gw, const uint32_t* __r
   for (int q = 0; q < C::S; q++) k[q] = dw[q];
   xyzz_mul_words<C>(R, G, k, C::S);
   store_xyzz<C>(out2 + XW, R);
+}
+
+// uniform-ish scalars in [0, r) for the small-n window-size autotune (engine.cu): hashed
+// words, the top word reduced below r's top word
+template <class C>
+__global__ void k_rand_scalars(uint32_t* __restrict__ out, size_t n, uint32_t seed) {
+  const size_t i = (size_t)blockIdx.x * blockDim.x + threadIdx.x;
+  if (i >= n) return;
+  for (int q = 0; q < C::S; q++) {
+    uint32_t x = (uint32_t)i * 0x9E3779B9u ^ (uint32_t)(i >> 32) * 0xC2B2AE35u ^ (uint32_t)q * 0x85EBCA6Bu ^ seed;
+    x ^= x >> 16; x *= 0x7feb352du; x ^= x >> 15; x *= 0x846ca68bu; x ^= x >> 16;
+    out[i * C::S + q] = q == C::S - 1 ? x % C::R32c()[C::S - 1] : x;
+  }
 }
 
 // thread t generates points [t*chunk, min((t+1)*chunk, n)) as canonical affine words

@@ -157,9 +157,10 @@ struct Ops final : CurveOps {
     uint32_t seg = o.seg > 0 ? (uint32_t)o.seg : (uint32_t)std::max<size_t>(4, cdiv((size_t)s.nset * nb, resident2));
     s.seg = seg;
     s.nseg = (uint32_t)cdiv(nb, seg);
-    // latency-mode products (k_bucket_segments<C, true>): measured slower even below half a
-    // wave (C1 reduce 0.253 -> 0.269 ms, C2 1.073 -> 1.126 ms), so off; kept as an A/B
-    s.seg_lat = 0;
+    // small n (segments below half a wave): k_bucket_segments<C, true> would run the
+    // call-based PADD (MSM_UNI_ALL A/B, measured slower) — off; r01's latency-mode products
+    // (LAT without MSM_UNI_ALL) measured slower too (C1 reduce 0.253 -> 0.269 ms)
+    s.seg_lat = (MSM_UNI_ALL && (size_t)s.nset * s.nseg * 2 < resident2) ? 1 : 0;
     if (!pre) free_table(s);
     else if (!s.table || s.table_c != c) {
       free_table(s);
@@ -205,7 +206,14 @@ struct Ops final : CurveOps {
       const int rest = KB - b3;
       s.s3_b2 = std::min(9, rest / 2);
       s.s3_b1 = rest - s.s3_b2;
+      // P1 keys are the flat key's low b2 + b3 bits: u16 when <= 16 (move bits into b1 if it
+      // has room; b2 only shrinks, so b2 <= 9 still holds)
+      if (s.s3_b2 + b3 > 16 && KB - 16 <= 9) {
+        s.s3_b1 = KB - 16;
+        s.s3_b2 = rest - s.s3_b1;
+      }
       s.s3_b3 = b3;
+      s.s3_k16 = s.s3_b2 + b3 <= 16 ? 1 : 0;
       const size_t NC1 = (size_t)1 << s.s3_b1, NC2 = (size_t)1 << s.s3_b2;
       dalloc(&s.s3Count, NC1);
       dalloc(&s.s3Off, NC1 + 1);
@@ -218,8 +226,10 @@ struct Ops final : CurveOps {
       dalloc(&s.s3v1, Mmax);
       dalloc(&s.s3k2, Mmax);
       dalloc(&s.s3v2, Mmax);
-      CK(cudaFuncSetAttribute(k_s3_part1<C>, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * S3_TILE * 4));
-      CK(cudaFuncSetAttribute(k_s3_part2, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * S3_TILE * 4));
+      CK(cudaFuncSetAttribute(k_s3_part1<C, uint16_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * S3_TILE * 4));
+      CK(cudaFuncSetAttribute(k_s3_part1<C, uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * S3_TILE * 4));
+      CK(cudaFuncSetAttribute(k_s3_part2<uint16_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * S3_TILE * 4));
+      CK(cudaFuncSetAttribute(k_s3_part2<uint32_t>, cudaFuncAttributeMaxDynamicSharedMemorySize, 2 * S3_TILE * 4));
       CK(cudaFuncSetAttribute(k_s3_part3, cudaFuncAttributeMaxDynamicSharedMemorySize, (S3_CAP + S3_MAXFINE) * 4));
     }
     if (s.sort_mode == 4) {
@@ -244,11 +254,27 @@ struct Ops final : CurveOps {
   }
 
   int enqueue_pipeline(Shard& s, const uint32_t* scal, bool timed) override {
+    return enqueue_range(s, scal, s.n, 0, false, true, s.goff, timed);
+  }
+
+  // Chunked host scalars (engine.cu): chunk k of the shard's points [ibase, ibase + n)
+  // is sorted and accumulated INTO the bucket set (zeroed before chunk 0; INIT
+  // accumulation from chunk 1 on), so its H2D overlaps the previous chunk's work; the
+  // last chunk runs the bucket reduce over every bucket (goff = nullptr) and a6.
+  bool can_chunk(const Shard& s) const override {
+    return kAccSync && !s.baff && (s.sort_mode == 3 || s.sort_mode == 4) && MSM_ACC_SMEM == 0;
+  }
+  int enqueue_chunk(Shard& s, const uint32_t* scal, size_t n, size_t ibase, bool first, bool last, bool timed) override {
+    if (first) CK(cudaMemsetAsync(s.buckets, 0, s.F * XW_ * sizeof(uint32_t), s.stream));
+    return enqueue_range(s, scal, n, (uint32_t)ibase, !first, last, nullptr, timed);
+  }
+
+  int enqueue_range(Shard& s, const uint32_t* scal, size_t n, uint32_t ibase, bool init, bool reduce,
+                    const uint32_t* red_goff, bool timed) {
     cudaStream_t st = s.stream;
     int launches = 0;
-    const size_t n = s.n;
     // flat-bucket / flat-bin stride per window and table-row stride (f3: one shared set)
-    const uint32_t ws = s.pre ? 0u : s.NB, wsb = s.pre ? 0u : s.nbin, istride = s.pre ? (uint32_t)n : 0u;
+    const uint32_t ws = s.pre ? 0u : s.NB, wsb = s.pre ? 0u : s.nbin, istride = s.pre ? (uint32_t)s.n : 0u;  // table row stride (all points of the shard)
     const uint32_t* pts = s.pre ? s.table : s.pts;
     if (timed) CK(cudaEventRecord(s.ev[EV_H2D], st));
     // a2 + a3: digits, histogram, scan, scatter
@@ -270,7 +296,7 @@ struct Ops final : CurveOps {
         const uint32_t tp = std::max<uint32_t>(1, s4_t1(NC1) / (uint32_t)s.nwin);
         const size_t ctas = cdiv(cdiv(n, tp), S4_CL) * S4_CL;
         k_s4_part1<C><<<(unsigned)ctas, S4_THREADS, 12 * NC1 + 14 * s4_t1(NC1), st>>>(
-            scal, n, s.c_arg, s.nwin, ws, istride, b2, NC1, tp, s.s4Cursor, s.s4k, s.s4v);
+            scal, n, s.c_arg, s.nwin, ws, istride, b2, NC1, tp, s.s4Cursor, s.s4k, s.s4v, ibase);
         launches++;
       }
       CK(cudaMemcpyAsync(s.goff + s.F, s.s4Off + NC1, 4, cudaMemcpyDeviceToDevice, st));
@@ -292,23 +318,36 @@ struct Ops final : CurveOps {
       k_scan_apply<<<(unsigned)nt, SCAN_THREADS, 0, st>>>(s.s3Count, NC1, s.tiles, s.s3Off, s.s3Cursor);
       launches += 3;
       const uint32_t tp = (uint32_t)std::max(1, S3_TILE / s.nwin);
+      uint16_t* k1s = reinterpret_cast<uint16_t*>(s.s3k1);
+      uint16_t* k2s = reinterpret_cast<uint16_t*>(s.s3k2);
       if (n) {
-        k_s3_part1<C><<<(unsigned)cdiv(n, tp), S3_THREADS, 2 * S3_TILE * 4, st>>>(scal, n, s.c_arg, s.nwin, ws, istride, sh1,
-                                                                                NC1, tp, s.s3Cursor, s.s3k1, s.s3v1);
+        if (s.s3_k16)
+          k_s3_part1<C, uint16_t><<<(unsigned)cdiv(n, tp), S3_THREADS, 2 * S3_TILE * 4, st>>>(
+              scal, n, s.c_arg, s.nwin, ws, istride, sh1, NC1, tp, s.s3Cursor, k1s, s.s3v1, ibase);
+        else
+          k_s3_part1<C, uint32_t><<<(unsigned)cdiv(n, tp), S3_THREADS, 2 * S3_TILE * 4, st>>>(
+              scal, n, s.c_arg, s.nwin, ws, istride, sh1, NC1, tp, s.s3Cursor, s.s3k1, s.s3v1, ibase);
         launches++;
       }
-      const unsigned maxTiles = (unsigned)(cdiv(std::max<size_t>(s.n * (size_t)s.nwin, 1), S3_TILE) + NC1);
+      const unsigned maxTiles = (unsigned)(cdiv(std::max<size_t>(n * (size_t)s.nwin, 1), S3_TILE) + NC1);
       const size_t nsub = (size_t)NC1 * NC2, nts = cdiv(nsub, SCAN_TILE);
       k_s3_tiles<<<1, S3_THREADS, 0, st>>>(s.s3Off, NC1, s.s3Tiles);
       CK(cudaMemsetAsync(s.s3SubCount, 0, nsub * sizeof(uint32_t), st));
-      k_s3_count2<<<maxTiles, S3_THREADS, 0, st>>>(s.s3Tiles, s.s3Off, NC1, s.s3_b3, NC2, s.s3k1, s.s3SubCount);
+      if (s.s3_k16)
+        k_s3_count2<uint16_t><<<maxTiles, S3_THREADS, 0, st>>>(s.s3Tiles, s.s3Off, NC1, s.s3_b3, NC2, k1s, s.s3SubCount);
+      else
+        k_s3_count2<uint32_t><<<maxTiles, S3_THREADS, 0, st>>>(s.s3Tiles, s.s3Off, NC1, s.s3_b3, NC2, s.s3k1, s.s3SubCount);
       k_scan_reduce<<<(unsigned)nts, SCAN_THREADS, 0, st>>>(s.s3SubCount, nsub, s.tiles);
       k_scan_tiles<<<1, 1024, 0, st>>>(s.tiles, nts, s.s3Sub + nsub);
       k_scan_apply<<<(unsigned)nts, SCAN_THREADS, 0, st>>>(s.s3SubCount, nsub, s.tiles, s.s3Sub, s.s3SubCursor);
-      k_s3_part2<<<maxTiles, S3_THREADS, 2 * S3_TILE * 4, st>>>(s.s3Tiles, s.s3Off, NC1, s.s3_b3, NC2, s.s3k1, s.s3v1,
-                                                                s.s3SubCursor, s.s3k2, s.s3v2);
+      if (s.s3_k16)
+        k_s3_part2<uint16_t><<<maxTiles, S3_THREADS, 2 * S3_TILE * 4, st>>>(s.s3Tiles, s.s3Off, NC1, s.s3_b3, NC2, k1s,
+                                                                            s.s3v1, s.s3SubCursor, k2s, s.s3v2);
+      else
+        k_s3_part2<uint32_t><<<maxTiles, S3_THREADS, 2 * S3_TILE * 4, st>>>(s.s3Tiles, s.s3Off, NC1, s.s3_b3, NC2, s.s3k1,
+                                                                            s.s3v1, s.s3SubCursor, k2s, s.s3v2);
       CK(cudaMemcpyAsync(s.goff + s.F, s.s3Off + NC1, 4, cudaMemcpyDeviceToDevice, st));
-      k_s3_part3<<<(unsigned)nsub, 256, (S3_CAP + (1u << s.s3_b3)) * 4, st>>>(s.s3Sub, s.s3_b3, (uint32_t)s.F, s.s3k2,
+      k_s3_part3<<<(unsigned)nsub, 256, (S3_CAP + (1u << s.s3_b3)) * 4, st>>>(s.s3Sub, s.s3_b3, (uint32_t)s.F, k2s,
                                                                              s.s3v2, s.goff, s.sorted);
       launches += 7;
     } else if (s.sort_mode == 2) {
@@ -373,7 +412,10 @@ struct Ops final : CurveOps {
     k_accumulate_smem<C><<<(unsigned)cdiv(s.acc_threads, 128), 128, ACC_SLOTS * C::L * ACC_NT * 4, st>>>(pts, s.sorted, s.goff, (uint32_t)s.F,
 #else
     if constexpr (kAccSync) {
-      if (s.baff)
+      if (init)
+        k_accumulate_sync<C, false, true><<<(unsigned)cdiv(s.acc_threads, ACC_SYNC_NT), ACC_SYNC_NT, 0, st>>>(
+            pts, s.sorted, s.goff, (uint32_t)s.F, s.buckets, s.carry_pts, s.carry_f, s.acc_threads, s.nlong);
+      else if (s.baff)
         k_accumulate_sync<C, true><<<(unsigned)cdiv(s.acc_threads, ACC_SYNC_NT), ACC_SYNC_NT, 0, st>>>(
             acc_pts, s.sorted, acc_goff, (uint32_t)s.F, s.buckets, s.carry_pts, s.carry_f, s.acc_threads, s.nlong);
       else
@@ -394,14 +436,15 @@ struct Ops final : CurveOps {
     launches += 2;
     CK(cudaGetLastError());
     if (timed) CK(cudaEventRecord(s.ev[EV_FIX], st));
+    if (!reduce) return launches;
     // a5: bucket reduce
     const uint32_t total = (uint32_t)s.nset * s.nseg;
     if (s.seg_lat)
       k_bucket_segments<C, true><<<(unsigned)cdiv(total, SEG_NT), SEG_NT, 0, st>>>(
-          s.buckets, s.goff, s.nset, s.NB, s.seg, s.nseg, (uint32_t)s.split_G, (uint32_t)s.split_g, s.segA);
+          s.buckets, red_goff, s.nset, s.NB, s.seg, s.nseg, (uint32_t)s.split_G, (uint32_t)s.split_g, s.segA);
     else
       k_bucket_segments<C, false><<<(unsigned)cdiv(total, SEG_NT), SEG_NT, 0, st>>>(
-          s.buckets, s.goff, s.nset, s.NB, s.seg, s.nseg, (uint32_t)s.split_G, (uint32_t)s.split_g, s.segA);
+          s.buckets, red_goff, s.nset, s.NB, s.seg, s.nseg, (uint32_t)s.split_G, (uint32_t)s.split_g, s.segA);
     launches++;
     uint32_t nin = s.nseg;
     uint32_t* src = s.segA;
@@ -508,6 +551,12 @@ struct Ops final : CurveOps {
     CK(cudaStreamSynchronize(s.stream));
     dfree(d);
     return (long)h;
+  }
+
+  void rand_scalars(Shard& s, uint32_t* out, size_t n, uint32_t seed) override {
+    if (!n) return;
+    k_rand_scalars<C><<<(unsigned)cdiv(n, 128), 128, 0, s.stream>>>(out, n, seed);
+    CK(cudaGetLastError());
   }
 
   void to_affine(const uint32_t* in, size_t n, uint32_t* out, cudaStream_t st) override {

@@ -48,6 +48,17 @@ struct Shard {
   size_t off = 0, n = 0;
   cudaStream_t stream = nullptr;
   cudaEvent_t ev[EV_COUNT] = {};
+  // chunked host scalars: copy stream and one event per chunk (created on first use)
+  cudaStream_t cstream = nullptr;
+  cudaEvent_t cev[8] = {};
+  int chunks_used = 1;
+  // small-n launch path: a2..a6 captured once into a CUDA graph and replayed while the
+  // configuration (gen) and the device scalar pointer stay the same (engine.cu)
+  cudaGraph_t graph = nullptr;
+  cudaGraphExec_t gexec = nullptr;
+  const uint32_t* g_scal = nullptr;
+  const uint32_t* last_scal = nullptr;
+  int gen = 0, g_gen = -1, g_launches = 0;
   // configuration (depends on c)
   int c = 0, nwin = 0;
   int pre = 0;         // precomputed window table in use (f3): one bucket set for all windows
@@ -77,6 +88,7 @@ struct Shard {
   uint16_t* binFine = nullptr;
   // three-level staged sort (sort3.cuh): key bits b1 + b2 + b3 >= bits(F - 1)
   int s3_b1 = 0, s3_b2 = 0, s3_b3 = 0;
+  int s3_k16 = 0;  // P1 keys as u16 (b2 + b3 <= 16)
   uint32_t *s3Count = nullptr, *s3Off = nullptr, *s3Cursor = nullptr, *s3Sub = nullptr,
            *s3k1 = nullptr, *s3v1 = nullptr, *s3k2 = nullptr, *s3v2 = nullptr, *s3SubCount = nullptr,
            *s3SubCursor = nullptr, *s3Tiles = nullptr;
@@ -105,6 +117,8 @@ struct Options {
   int pre = 2;   // f3 precomputation: 0 off, 1 on, 2 auto (on when the table fits in memory)
   int split_G = 1, split_g = 0;  // f1: this context sums only buckets |d| = G*q + g
   int acc_mode = 2;  // a4: 0 PACC only, 1 batch-affine front end + PACC (ablation), 2 auto (= 0, measured faster)
+  int chunks = 0;    // host-scalar H2D chunks per msm_run: 0 auto, 1 one copy, K >= 2 (engine.cu)
+  int tuned_c = 0;   // window size measured best at context creation (small n, c auto; engine.cu)
 };
 
 // Per-curve kernels behind a virtual interface (one instance per curve, curve_*.cu).
@@ -124,6 +138,11 @@ struct CurveOps {
   // enqueue a2..a6 on s.stream for the shard's scalars; the partial ends in s.partial.
   // Returns the number of kernels launched.
   virtual int enqueue_pipeline(Shard& s, const uint32_t* scal_dev, bool timed) = 0;
+  // chunked host scalars: whether this shard's configuration supports it, and one chunk
+  // (points [ibase, ibase + n) of the shard, scalars already on the device at scal_dev)
+  virtual bool can_chunk(const Shard& s) const = 0;
+  virtual int enqueue_chunk(Shard& s, const uint32_t* scal_dev, size_t n, size_t ibase, bool first, bool last,
+                            bool timed) = 0;
   virtual void enqueue_finalize(const uint32_t* partials_dev, int count, uint32_t* result_dev, cudaStream_t st) = 0;
   virtual void gen_points(const uint32_t* e0, const uint32_t* delta, size_t n, uint32_t* out) = 0;
   virtual void debug_field(int op, const uint32_t* a, const uint32_t* b, size_t n, uint32_t* out) = 0;
@@ -132,6 +151,7 @@ struct CurveOps {
   virtual void to_affine(const uint32_t* in_dev, size_t n, uint32_t* out_dev, cudaStream_t st) = 0;
   virtual long count_nonempty(Shard& s) = 0;
   virtual bool has_baff() const = 0;
+  virtual void rand_scalars(Shard& s, uint32_t* out_dev, size_t n, uint32_t seed) = 0;
 };
 
 inline int num_windows(int lambda, int c) { return lambda / c + 1; }

@@ -14,7 +14,8 @@
 //                    from a global scan of the per-(bin, sub-bin) counts);
 //   P3  k_s3_part3   one block per sub-bin (2^b3 buckets, ~4-8K entries): a complete
 //                    counting sort in shared memory, written contiguously, plus goff.
-// The (i, j) entry value is (i + j*istride) | sign<<31 as in the other sort variants.
+// The (i, j) entry value is (i + j*istride) | sign<<31 as in the other sort variants (i
+// offset by ibase when the scalars arrive in chunks: engine.cu, chunked host H2D).
 // Why: the two-level binned sort (k_bin_scatter) wrote 6-B entries at random positions
 // of 8K bins; ncu measured 28.7 GB DRAM writes for 4.4 GB of entries at 2^26 (partial
 // sectors evicted before they fill) -- 31 ms of a 40 ms sort.
@@ -29,29 +30,29 @@ constexpr int S3_MAXFINE = 4096;     // max buckets per sub-bin (b3 <= 12)
 // P2/P3 passes were global-load-latency bound (ncu: long_scoreboard ~35-49 stalls per
 // issue, 14-17 % issue) with one key load outstanding per thread.
 constexpr int S3_U = 8;
-template <class F>
-__device__ __forceinline__ void s3_for_keys(const uint32_t* __restrict__ keys, uint32_t e0, uint32_t e1, F&& f) {
+template <class KT, class F>
+__device__ __forceinline__ void s3_for_keys(const KT* __restrict__ keys, uint32_t e0, uint32_t e1, F&& f) {
   for (uint32_t eb = e0 + threadIdx.x; eb < e1; eb += S3_U * blockDim.x) {
     uint32_t k[S3_U];
 #pragma unroll
     for (int u = 0; u < S3_U; u++) {
       const uint32_t e = eb + u * blockDim.x;
-      k[u] = e < e1 ? __ldg(keys + e) : 0u;
+      k[u] = e < e1 ? (uint32_t)__ldg(keys + e) : 0u;
     }
 #pragma unroll
     for (int u = 0; u < S3_U; u++)
       if (eb + u * blockDim.x < e1) f(k[u]);
   }
 }
-template <class F>
-__device__ __forceinline__ void s3_for_entries(const uint32_t* __restrict__ keys, const uint32_t* __restrict__ vals,
+template <class KT, class F>
+__device__ __forceinline__ void s3_for_entries(const KT* __restrict__ keys, const uint32_t* __restrict__ vals,
                                                uint32_t e0, uint32_t e1, F&& f) {
   for (uint32_t eb = e0 + threadIdx.x; eb < e1; eb += S3_U * blockDim.x) {
     uint32_t k[S3_U], v[S3_U];
 #pragma unroll
     for (int u = 0; u < S3_U; u++) {
       const uint32_t e = eb + u * blockDim.x;
-      k[u] = e < e1 ? __ldg(keys + e) : 0u;
+      k[u] = e < e1 ? (uint32_t)__ldg(keys + e) : 0u;
       v[u] = e < e1 ? __ldg(vals + e) : 0u;
     }
 #pragma unroll
@@ -103,11 +104,14 @@ __global__ void __launch_bounds__(S3_THREADS) k_s3_count1(const uint32_t* __rest
 }
 
 // P1: tile = tp points (tp * nwin <= S3_TILE entries)
-template <class C>
+// KT: P1 keys leave as the flat key's low sh1 bits (the bin is the position), u16 when
+// sh1 <= 16 (round 2: 6 instead of 8 bytes per entry through P2)
+template <class C, class KT>
 __global__ void __launch_bounds__(S3_THREADS) k_s3_part1(const uint32_t* __restrict__ scal, size_t n, int c, int nwin,
                                                          uint32_t ws, uint32_t istride, int sh1, uint32_t NC1, uint32_t tp,
                                                          uint32_t* __restrict__ binCursor,
-                                                         uint32_t* __restrict__ keys, uint32_t* __restrict__ vals) {
+                                                         KT* __restrict__ keys, uint32_t* __restrict__ vals,
+                                                         uint32_t ibase = 0) {
   extern __shared__ uint32_t sm[];
   uint32_t* skey = sm;                 // [S3_TILE]
   uint32_t* sval = sm + S3_TILE;       // [S3_TILE]
@@ -140,14 +144,15 @@ __global__ void __launch_bounds__(S3_THREADS) k_s3_part1(const uint32_t* __restr
       const uint32_t f = j * ws + b;
       const uint32_t pos = atomicAdd(cur + (f >> sh1), 1u);
       skey[pos] = f;
-      sval[pos] = ((uint32_t)i + (uint32_t)j * istride) | (neg ? SIGN_BIT : 0u);
+      sval[pos] = ((uint32_t)i + ibase + (uint32_t)j * istride) | (neg ? SIGN_BIT : 0u);
     });
   }
   __syncthreads();
+  const uint32_t lowmask = sh1 >= 32 ? ~0u : (1u << sh1) - 1u;
   for (uint32_t p = threadIdx.x; p < E; p += blockDim.x) {
     const uint32_t f = skey[p], bin = f >> sh1;
     const uint32_t o = gbase[bin] + (p - loc[bin]);
-    keys[o] = f;
+    keys[o] = (KT)(f & lowmask);
     vals[o] = sval[p];
   }
 }
@@ -182,10 +187,11 @@ __device__ __forceinline__ bool s3_tile(const uint32_t* __restrict__ tileStart, 
 }
 
 // P2 histogram: subCount[bin*NC2 + s] for s = (f >> sh2) & (NC2 - 1)
-static __global__ void __launch_bounds__(S3_THREADS) k_s3_count2(const uint32_t* __restrict__ tileStart,
-                                                                 const uint32_t* __restrict__ binOff, uint32_t NC1,
-                                                                 int sh2, uint32_t NC2, const uint32_t* __restrict__ keys,
-                                                                 uint32_t* __restrict__ subCount) {
+template <class KT>
+__global__ void __launch_bounds__(S3_THREADS) k_s3_count2(const uint32_t* __restrict__ tileStart,
+                                                          const uint32_t* __restrict__ binOff, uint32_t NC1,
+                                                          int sh2, uint32_t NC2, const KT* __restrict__ keys,
+                                                          uint32_t* __restrict__ subCount) {
   __shared__ uint32_t hist[S3_MAXB];
   uint32_t bin, e0, e1;
   if (!s3_tile(tileStart, binOff, NC1, blockIdx.x, bin, e0, e1)) return;
@@ -200,12 +206,14 @@ static __global__ void __launch_bounds__(S3_THREADS) k_s3_count2(const uint32_t*
 
 // P2 scatter: per tile, shared-memory ranks by sub-bin, one global atomic per (tile,
 // sub-bin) on subCursor (initialised to the global sub-bin starts), staged coalesced runs.
-static __global__ void __launch_bounds__(S3_THREADS) k_s3_part2(const uint32_t* __restrict__ tileStart,
-                                                                const uint32_t* __restrict__ binOff, uint32_t NC1,
-                                                                int sh2, uint32_t NC2,
-                                                                const uint32_t* __restrict__ keys, const uint32_t* __restrict__ vals,
-                                                                uint32_t* __restrict__ subCursor,
-                                                                uint32_t* __restrict__ keys2, uint32_t* __restrict__ vals2) {
+// P2 keys leave as the low sh2 = b3 bits (u16; b3 <= 12)
+template <class KT>
+__global__ void __launch_bounds__(S3_THREADS) k_s3_part2(const uint32_t* __restrict__ tileStart,
+                                                         const uint32_t* __restrict__ binOff, uint32_t NC1,
+                                                         int sh2, uint32_t NC2,
+                                                         const KT* __restrict__ keys, const uint32_t* __restrict__ vals,
+                                                         uint32_t* __restrict__ subCursor,
+                                                         uint16_t* __restrict__ keys2, uint32_t* __restrict__ vals2) {
   extern __shared__ uint32_t sm[];
   uint32_t* skey = sm;
   uint32_t* sval = sm + S3_TILE;
@@ -232,10 +240,11 @@ static __global__ void __launch_bounds__(S3_THREADS) k_s3_part2(const uint32_t* 
     sval[pos] = v;
   });
   __syncthreads();
+  const uint32_t lowmask = (1u << sh2) - 1u;
   for (uint32_t p = threadIdx.x; p < E; p += blockDim.x) {
     const uint32_t f = skey[p], sb = (f >> sh2) & mask;
     const uint32_t o = gbase[sb] + (p - loc[sb]);
-    keys2[o] = f;
+    keys2[o] = (uint16_t)(f & lowmask);
     vals2[o] = sval[p];
   }
 }
@@ -243,7 +252,7 @@ static __global__ void __launch_bounds__(S3_THREADS) k_s3_part2(const uint32_t* 
 // P3: block = sub-bin q covering buckets [q << b3, (q+1) << b3) of [subOff[q], end_q);
 // writes goff for its buckets (< F) and the final values in bucket order.
 static __global__ void __launch_bounds__(256) k_s3_part3(const uint32_t* __restrict__ subOff, int b3, uint32_t F,
-                                                         const uint32_t* __restrict__ keys2, const uint32_t* __restrict__ vals2,
+                                                         const uint16_t* __restrict__ keys2, const uint32_t* __restrict__ vals2,
                                                          uint32_t* __restrict__ goff, uint32_t* __restrict__ sorted) {
   extern __shared__ uint32_t sm[];
   uint32_t* sval = sm;                  // [S3_CAP] staged values (bucket order)

@@ -82,7 +82,7 @@ template <class C>
 __global__ void __cluster_dims__(S4_CL, 1, 1) __launch_bounds__(S4_THREADS, 1)
     k_s4_part1(const uint32_t* __restrict__ scal, size_t n, int cp, int nwin, uint32_t ws, uint32_t istride, int b2,
                uint32_t NC1, uint32_t tp, uint32_t* __restrict__ binCursor, uint16_t* __restrict__ keys,
-               uint32_t* __restrict__ vals) {
+               uint32_t* __restrict__ vals, uint32_t ibase = 0) {
   extern __shared__ uint32_t sm[];
   const uint32_t T1 = s4_t1(NC1);
   uint32_t* cnt = sm;              // [NC1] local counts (read remotely), then local bin starts
@@ -144,7 +144,7 @@ __global__ void __cluster_dims__(S4_CL, 1, 1) __launch_bounds__(S4_THREADS, 1)
     const uint32_t pl = nwin == 1 ? s : __umulhi(s, magic);
     const uint32_t j = s - pl * (uint32_t)nwin;
     Tk[pos] = fb;
-    Tv[pos] = ((uint32_t)(p0 + pl) + j * istride) | (f & SIGN_BIT);
+    Tv[pos] = ((uint32_t)(p0 + pl) + ibase + j * istride) | (f & SIGN_BIT);
   }
   __syncthreads();
   const uint32_t mask = (1u << b2) - 1u;
@@ -204,7 +204,7 @@ __device__ __forceinline__ void s4_cluster_scan(cg::cluster_group& cl, uint32_t*
 }
 
 // P2: cluster b = bin b, buckets f in [b << b2, (b+1) << b2) (those < F get goff).
-__global__ void __cluster_dims__(S4_CL, 1, 1) __launch_bounds__(S4_THREADS2, 1)
+static __global__ void __cluster_dims__(S4_CL, 1, 1) __launch_bounds__(S4_THREADS2, 1)
     k_s4_part2(const uint32_t* __restrict__ binOff, int b2, uint32_t F, const uint16_t* __restrict__ keys,
                const uint32_t* __restrict__ vals, uint32_t* __restrict__ goff, uint32_t* __restrict__ sorted) {
   extern __shared__ uint32_t sm[];

@@ -388,6 +388,7 @@ def test_bucket_split_large_balanced(lib):
     entries = []
     for g in range(G):
         ctx = lib.Context(name, pts, n=n)
+        ctx.set_option(lib.OPT_WINDOW_BITS, 14)  # the cost model's c (creation autotunes small n)
         ctx.set_option(lib.OPT_SPLIT_PARTS, G)
         ctx.set_option(lib.OPT_SPLIT_INDEX, g)
         ctx.run_partial(ks, parts[g * pw:(g + 1) * pw])

@@ -221,3 +221,57 @@ def test_cluster_sort_heavy_bins(lib, kind, cbits, pre):
         assert ctx.run(ks_w) == want
     finally:
         ctx.close()
+
+
+@pytest.mark.parametrize("pre", [1, 0])
+def test_chunked_host_scalars(lib, pre):
+    """Host scalars uploaded in K growing chunks, each sorted and accumulated INTO the
+    bucket set (INIT accumulation): bit-exact against the closed form for
+    K = 1..5 (and auto = 3), with the f3 table on and off, BLS12-381 n = 2^20; device
+    scalars are never chunked."""
+    name = "bls12_381"
+    c = CURVES[name]
+    n = 1 << 20
+    pts, es = gen_device_points(lib, name, n, 80)
+    ks_w = synth.scalars_range(c.r, 0, n, 81)
+    ks = synth.words_to_ints(ks_w)
+    ks_w[5] = 0                       # a zero scalar inside the first chunk
+    ks[5] = 0
+    want = ec.to_output(ec.mul(sum(k * e for k, e in zip(ks, es)) % c.r, c.G, c))
+    ctx = lib.Context(name, pts, n=n)
+    try:
+        ctx.set_option(lib.OPT_PRECOMPUTE, pre)
+        for K, used in ((0, 3), (1, 1), (2, 2), (4, 4), (5, 5)):
+            ctx.set_option(lib.OPT_H2D_CHUNKS, K)
+            assert ctx.run(ks_w) == want, K
+            assert ctx.get_option(lib.OPT_H2D_CHUNKS) == used
+        import torch
+        assert ctx.run(torch.from_numpy(ks_w.view(np.int32)).cuda()) == want
+        assert ctx.get_option(lib.OPT_H2D_CHUNKS) == 1
+    finally:
+        ctx.close()
+
+
+def test_small_n_autotune(lib):
+    """Contexts of 2^10..2^17 points with automatic c measure the candidate window sizes at
+    creation and keep the fastest (engine.cu autotune_c): the chosen c is one of the
+    candidates, results stay bit-exact, and an explicit c still wins over the tuned one."""
+    name = "bn254"
+    c = CURVES[name]
+    n = 1 << 12
+    pts, es = gen_device_points(lib, name, n, 90)
+    ks_w = synth.scalars_range(c.r, 0, n, 91)
+    ks = synth.words_to_ints(ks_w)
+    want = ec.to_output(ec.mul(sum(k * e for k, e in zip(ks, es)) % c.r, c.G, c))
+    ctx = lib.Context(name, pts, n=n)
+    try:
+        tuned = ctx.get_option(lib.OPT_WINDOW_BITS)
+        assert 4 <= tuned <= 16
+        assert ctx.run(ks_w) == want
+        ctx.set_option(lib.OPT_WINDOW_BITS, 9)
+        assert ctx.get_option(lib.OPT_WINDOW_BITS) == 9
+        assert ctx.run(ks_w) == want
+        ctx.set_option(lib.OPT_WINDOW_BITS, 0)
+        assert ctx.get_option(lib.OPT_WINDOW_BITS) == tuned
+    finally:
+        ctx.close()
