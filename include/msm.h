@@ -108,10 +108,14 @@ enum {
                                  ...) on a copy stream, each sorted and accumulated INTO the
                                  bucket set while the next one uploads ("can be
                                  efficiently pipelined"); 0 = auto (default: K = 3 for
-                                 n >= 2^20 per shard where supported: BN254, BLS12-377/381 with
+                                 n >= 2^22 per shard where supported: BN254, BLS12-377/381 with
                                  the staged or cluster sort), 1 = one copy before the MSM,
                                  2..8 = K.  Device scalars are never chunked.  Get returns the
                                  K used by the last run on shard 0.  No reconfiguration.      */
+  MSM_OPT_GRAPH = 10,         /* 1 (default) = shards of <= 2^17 points with device scalars
+                                 replay a2..a6 as a CUDA graph once the same scalar buffer is
+                                 seen twice (the stage times of such runs read -1 in
+                                 msm_stats, the total stays valid); 0 = always launch kernels */
   MSM_OPT_NWIN = 101,         /* (get only) number of windows floor(lambda/c) + 1           */
   MSM_OPT_NSETS = 103,        /* (get only) bucket sets: nwin, or 1 with the f3 table        */
   MSM_OPT_NONEMPTY = 102,     /* (get only) non-empty buckets of the last run on shard 0    */

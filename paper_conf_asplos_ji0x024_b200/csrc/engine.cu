@@ -44,6 +44,8 @@ struct msm_context {
   long next_ticket = 0, next_wait = 0;
   uint32_t* h_run = nullptr;     // pinned [2*L32 + 1]: msm_run's result and error word (one D2H)
   bool stats_pending = false;    // msm_stats of the last run are read lazily (msm_get_stats)
+  int graph = 1;                 // MSM_OPT_GRAPH: small-n CUDA-graph replay allowed
+  bool last_graphed = false;     // the last run replayed a graph: no per-stage events
 };
 
 namespace {
@@ -213,7 +215,9 @@ void destroy_shard(CurveOps* ops, Shard& s) {
 
 int apply_window_bits(msm_context* ctx) {
   Options o = ctx->opt;
-  if (o.c == 0 && o.tuned_c > 0) o.c = o.tuned_c;
+  // the tuned c is a timing result, so it may differ between processes: the f1 bucket split
+  // needs the same c (the same digits) in every part, so it keeps the deterministic model
+  if (o.c == 0 && o.tuned_c > 0 && o.split_G == 1) o.c = o.tuned_c;
   for (auto& s : ctx->shards) {
     int c = 0, pre = 0;
     plan_shard(o, s, ctx->ops->lambda(), ctx->ops->PW(), ctx->ops->XW(), &c, &pre,
@@ -329,7 +333,9 @@ const uint32_t* stage_scalars(msm_context* ctx, Shard& s, const uint32_t* scalar
 int h2d_chunks(msm_context* ctx, const Shard& s) {
   const int want = ctx->opt.chunks;
   if (want == 1 || s.n == 0 || !ctx->ops->can_chunk(s)) return 1;
-  if (want == 0) return s.n >= ((size_t)1 << 20) ? 3 : 1;
+  // auto: from 2^22 points (BLS12-377 2^24: 103.8 -> 99.0 ms; at 2^20 it is neutral,
+  // 9.28 vs 9.32 ms, profiles/r02b/configs.jsonl)
+  if (want == 0) return s.n >= ((size_t)1 << 22) ? 3 : 1;
   return std::min(want, 8);
 }
 
@@ -395,10 +401,14 @@ int run_all(msm_context* ctx, const uint32_t* scalars, bool gather_to_dev0) {
         const uint32_t* sc = stage_scalars(ctx, s, scalars, is_dev, src_dev);
         NvtxRange nr("enqueue a2..a6 (shard)");
         static const bool no_graph = getenv("MSM_NO_GRAPH") != nullptr;  // A/B
-        if (!no_graph && is_dev && src_dev == s.dev && s.n <= GRAPH_MAX_N && sc != s.scal)
+        bool graphed = false;
+        if (!no_graph && ctx->graph && is_dev && src_dev == s.dev && s.n <= GRAPH_MAX_N && sc != s.scal) {
           launched[g] = enqueue_graphed(ctx, s, sc, timed);
-        else
+          graphed = s.gexec && s.g_scal == sc && s.g_gen == s.gen;
+        } else {
           launched[g] = ctx->ops->enqueue_pipeline(s, sc, timed);
+        }
+        if (g == 0) ctx->last_graphed = graphed;
       }
     } catch (const CudaError& e) {
       rc[g] = e.code;
@@ -454,6 +464,8 @@ void collect_stats(msm_context* ctx) {
   st.fixup_ms = el(EV_ACC, EV_FIX);
   st.reduce_ms = el(EV_FIX, EV_RED);
   st.combine_ms = el(EV_RED, EV_COMB);
+  if (ctx->last_graphed)  // a replayed graph has no per-stage events: a2..a6 unknown (-1)
+    st.sort_ms = st.accumulate_ms = st.baff_ms = st.fixup_ms = st.reduce_ms = st.combine_ms = -1.0f;
   st.finalize_ms = el(EV_COMB, EV_END);
   st.total_ms = el(EV_START, EV_END);
   st.window_bits = s.c;
@@ -858,6 +870,10 @@ int msm_set_option(msm_context* ctx, int key, long value) {
       if (value < 0 || value > 8) return MSM_ERR_ARG;
       ctx->opt.chunks = (int)value;
       return MSM_OK;  // no reconfiguration
+    case MSM_OPT_GRAPH:
+      if (value < 0 || value > 1) return MSM_ERR_ARG;
+      ctx->graph = (int)value;
+      return MSM_OK;
     default:
       return MSM_ERR_ARG;
   }
@@ -878,6 +894,7 @@ long msm_get_option(msm_context* ctx, int key) {
     case MSM_OPT_SPLIT_INDEX: return ctx->opt.split_g;
     case MSM_OPT_ACC_MODE: return ctx->shards[0].baff;
     case MSM_OPT_H2D_CHUNKS: return ctx->shards[0].chunks_used;
+    case MSM_OPT_GRAPH: return ctx->graph;
     case MSM_OPT_DEVICE: return ctx->shards[0].dev;
     case MSM_OPT_NGPUS: return (long)ctx->shards.size();
     case MSM_OPT_NONEMPTY: {

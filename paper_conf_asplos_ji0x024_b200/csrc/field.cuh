@@ -259,8 +259,50 @@ DEVI void fmul_sum(uint32_t* r, const uint32_t* a, const uint32_t* b, const uint
   for (int i = 0; i < C::L; i++) r[i] = t[i];
 }
 
+#ifndef MSM_ROWS
+#define MSM_ROWS 0  // A/B: MNT4-753 products by operand scanning (fmul_rows) instead of columns
+#endif
+
+// Operand scanning with delayed carries, for the 27-limb field: row i adds a_i * b and
+// m_i * p into 64-bit column accumulators T[i..i+L) — L independent IMAD.WIDE chains per
+// row instead of one 54-deep chain per column (MNT4-753's accumulation is latency-bound:
+// r01 ncu "wait" 5.5 stalls per issue at 2 warps per scheduler).  m_i = T_i n'_0 mod 2^W
+// (T_i complete: every earlier row has added its terms and its carry), then T_{i+1} +=
+// T_i >> W.  A column gets <= 2L products of (2^W + 3)^2 plus carries < 2^35: < 2^64 for
+// W = 29, L = 27.  Same result and bounds as the column form.
+template <class C>
+DEVI void fmul_rows(uint32_t* r, const uint32_t* a, const uint32_t* b) {
+  constexpr int L = C::L, W = C::W;
+  constexpr uint32_t MASK = (1u << W) - 1;
+  u64 T[2 * L];
+#pragma unroll
+  for (int k = 0; k < 2 * L; k++) T[k] = 0;
+#pragma unroll
+  for (int i = 0; i < L; i++) {
+#pragma unroll
+    for (int j = 0; j < L; j++) T[i + j] = mad_wide(a[i], b[j], T[i + j]);
+    const uint32_t m = ((uint32_t)T[i] * C::N0) & MASK;
+#pragma unroll
+    for (int j = 0; j < L; j++)
+      if (C::P(j) != 0u) T[i + j] = mad_wide(m, C::P(j), T[i + j]);
+    T[i + 1] += T[i] >> W;
+  }
+  u64 c = 0;
+#pragma unroll
+  for (int k = 0; k < L - 1; k++) {
+    const u64 v = T[L + k] + c;
+    r[k] = (uint32_t)v & MASK;
+    c = v >> W;
+  }
+  r[L - 1] = (uint32_t)c;
+}
+
 template <class C, bool SQR, bool LAT = false>
 DEVI void fmul_impl(uint32_t* r, const uint32_t* a, const uint32_t* b) {
+  if constexpr (MSM_ROWS != 0 && C::L > 13) {
+    fmul_rows<C>(r, a, b);
+    return;
+  }
   constexpr int L = C::L;
   uint32_t m[L];
   uint32_t a2[L];
@@ -274,6 +316,11 @@ DEVI void fmul_impl(uint32_t* r, const uint32_t* a, const uint32_t* b) {
 // r1 = a1*b1, r2 = a2*b2 (SQR: r1 = a1^2, r2 = a2^2), same contract as fmul
 template <class C, bool SQR = false>
 DEVI void fmul2(uint32_t* r1, const uint32_t* a1, const uint32_t* b1, uint32_t* r2, const uint32_t* a2, const uint32_t* b2) {
+  if constexpr (MSM_ROWS != 0 && C::L > 13) {  // each product already has L-way ILP
+    fmul_rows<C>(r1, a1, b1);
+    fmul_rows<C>(r2, a2, b2);
+    return;
+  }
   constexpr int L = C::L;
   uint32_t m1[L], m2[L], d1[L], d2[L];
   if constexpr (SQR) {

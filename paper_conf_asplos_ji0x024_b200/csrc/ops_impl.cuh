@@ -11,6 +11,10 @@ namespace msmrt {
 
 using namespace msmk;
 
+#ifndef MSM_SEG_UNI
+#define MSM_SEG_UNI 0  // A/B (with MSM_UNI_ALL=1): call-based PADD in the bucket reduce at every n
+#endif
+
 template <class C>
 struct Ops final : CurveOps {
   // k_accumulate_sync (lockstep blocks, register-prefetched gathers) for L <= 13; MNT4-753
@@ -160,7 +164,7 @@ struct Ops final : CurveOps {
     // small n (segments below half a wave): k_bucket_segments<C, true> would run the
     // call-based PADD (MSM_UNI_ALL A/B, measured slower) — off; r01's latency-mode products
     // (LAT without MSM_UNI_ALL) measured slower too (C1 reduce 0.253 -> 0.269 ms)
-    s.seg_lat = (MSM_UNI_ALL && (size_t)s.nset * s.nseg * 2 < resident2) ? 1 : 0;
+    s.seg_lat = (MSM_UNI_ALL && (MSM_SEG_UNI || (size_t)s.nset * s.nseg * 2 < resident2)) ? 1 : 0;
     if (!pre) free_table(s);
     else if (!s.table || s.table_c != c) {
       free_table(s);

@@ -29,6 +29,7 @@ OPT_SPLIT_PARTS = 6
 OPT_SPLIT_INDEX = 7
 OPT_ACC_MODE = 8
 OPT_H2D_CHUNKS = 9
+OPT_GRAPH = 10
 OPT_NWIN = 101
 OPT_NONEMPTY = 102
 OPT_NSETS = 103

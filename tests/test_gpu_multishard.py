@@ -227,8 +227,8 @@ def test_cluster_sort_heavy_bins(lib, kind, cbits, pre):
 def test_chunked_host_scalars(lib, pre):
     """Host scalars uploaded in K growing chunks, each sorted and accumulated INTO the
     bucket set (INIT accumulation): bit-exact against the closed form for
-    K = 1..5 (and auto = 3), with the f3 table on and off, BLS12-381 n = 2^20; device
-    scalars are never chunked."""
+    K = 1..5 (auto = 1 below 2^22 points), with the f3 table on and off, BLS12-381
+    n = 2^20; device scalars are never chunked."""
     name = "bls12_381"
     c = CURVES[name]
     n = 1 << 20
@@ -241,7 +241,7 @@ def test_chunked_host_scalars(lib, pre):
     ctx = lib.Context(name, pts, n=n)
     try:
         ctx.set_option(lib.OPT_PRECOMPUTE, pre)
-        for K, used in ((0, 3), (1, 1), (2, 2), (4, 4), (5, 5)):
+        for K, used in ((0, 1), (1, 1), (2, 2), (3, 3), (4, 4), (5, 5)):  # auto: K = 3 from 2^22
             ctx.set_option(lib.OPT_H2D_CHUNKS, K)
             assert ctx.run(ks_w) == want, K
             assert ctx.get_option(lib.OPT_H2D_CHUNKS) == used
