@@ -161,10 +161,10 @@ struct Ops final : CurveOps {
     uint32_t seg = o.seg > 0 ? (uint32_t)o.seg : (uint32_t)std::max<size_t>(4, cdiv((size_t)s.nset * nb, resident2));
     s.seg = seg;
     s.nseg = (uint32_t)cdiv(nb, seg);
-    // small n (segments below half a wave): k_bucket_segments<C, true> would run the
-    // call-based PADD (MSM_UNI_ALL A/B, measured slower) — off; r01's latency-mode products
-    // (LAT without MSM_UNI_ALL) measured slower too (C1 reduce 0.253 -> 0.269 ms)
-    s.seg_lat = (MSM_UNI_ALL && (MSM_SEG_UNI || (size_t)s.nset * s.nseg * 2 < resident2)) ? 1 : 0;
+    // small n (segments below half a wave): k_bucket_segments<C, true> runs the shared
+    // out-of-line PADD body (MSM_SHARED_NI, ec.cuh); the call-based PADD (MSM_UNI_ALL) and
+    // r01's inline latency-mode products measured slower (C1 reduce 0.253 -> 0.269 ms)
+    s.seg_lat = ((MSM_UNI_ALL || MSM_SHARED_NI) && (MSM_SEG_UNI || (size_t)s.nset * s.nseg * 2 < resident2)) ? 1 : 0;
     if (!pre) free_table(s);
     else if (!s.table || s.table_c != c) {
       free_table(s);
@@ -411,22 +411,32 @@ struct Ops final : CurveOps {
       }
     }
     if (timed) CK(cudaEventRecord(s.ev[EV_BAFF], st));
+    // Small n: the accumulation and reduce threads are few (C1: ~2.8 K accumulation threads =
+    // 11 blocks of 256), and 8 warps of one SM then share its IMAD pipe while 137 SMs idle
+    // (ncu: 144 us for 17 PACC per thread).  Halve the block size (down to one warp) until the
+    // blocks cover the SMs.
+    auto spread = [&](size_t threads, uint32_t nt) {
+      uint32_t bs = nt;
+      while (bs > 32 && cdiv(std::max<size_t>(threads, 1), bs) < (size_t)s.sms) bs >>= 1;
+      return bs;
+    };
+    const uint32_t anb = spread(s.acc_threads, kAccSync ? ACC_SYNC_NT : 128);
     // a4: accumulate + fixup
 #if MSM_ACC_SMEM
     k_accumulate_smem<C><<<(unsigned)cdiv(s.acc_threads, 128), 128, ACC_SLOTS * C::L * ACC_NT * 4, st>>>(pts, s.sorted, s.goff, (uint32_t)s.F,
 #else
     if constexpr (kAccSync) {
       if (init)
-        k_accumulate_sync<C, false, true><<<(unsigned)cdiv(s.acc_threads, ACC_SYNC_NT), ACC_SYNC_NT, 0, st>>>(
+        k_accumulate_sync<C, false, true><<<(unsigned)cdiv(s.acc_threads, anb), anb, 0, st>>>(
             pts, s.sorted, s.goff, (uint32_t)s.F, s.buckets, s.carry_pts, s.carry_f, s.acc_threads, s.nlong);
       else if (s.baff)
-        k_accumulate_sync<C, true><<<(unsigned)cdiv(s.acc_threads, ACC_SYNC_NT), ACC_SYNC_NT, 0, st>>>(
+        k_accumulate_sync<C, true><<<(unsigned)cdiv(s.acc_threads, anb), anb, 0, st>>>(
             acc_pts, s.sorted, acc_goff, (uint32_t)s.F, s.buckets, s.carry_pts, s.carry_f, s.acc_threads, s.nlong);
       else
-        k_accumulate_sync<C><<<(unsigned)cdiv(s.acc_threads, ACC_SYNC_NT), ACC_SYNC_NT, 0, st>>>(
+        k_accumulate_sync<C><<<(unsigned)cdiv(s.acc_threads, anb), anb, 0, st>>>(
             pts, s.sorted, s.goff, (uint32_t)s.F, s.buckets, s.carry_pts, s.carry_f, s.acc_threads, s.nlong);
     } else
-      k_accumulate<C><<<(unsigned)cdiv(s.acc_threads, 128), 128, 0, st>>>(pts, s.sorted, s.goff, (uint32_t)s.F,
+      k_accumulate<C><<<(unsigned)cdiv(s.acc_threads, anb), anb, 0, st>>>(pts, s.sorted, s.goff, (uint32_t)s.F,
 #endif
                                                                         s.buckets, s.carry_pts, s.carry_f, s.acc_threads,
                                                                         s.nlong);
@@ -443,11 +453,12 @@ struct Ops final : CurveOps {
     if (!reduce) return launches;
     // a5: bucket reduce
     const uint32_t total = (uint32_t)s.nset * s.nseg;
+    const uint32_t snb = MSM_SEG_SYNC ? (uint32_t)SEG_NT : spread(total, SEG_NT);
     if (s.seg_lat)
-      k_bucket_segments<C, true><<<(unsigned)cdiv(total, SEG_NT), SEG_NT, 0, st>>>(
+      k_bucket_segments<C, true><<<(unsigned)cdiv(total, snb), snb, 0, st>>>(
           s.buckets, red_goff, s.nset, s.NB, s.seg, s.nseg, (uint32_t)s.split_G, (uint32_t)s.split_g, s.segA);
     else
-      k_bucket_segments<C, false><<<(unsigned)cdiv(total, SEG_NT), SEG_NT, 0, st>>>(
+      k_bucket_segments<C, false><<<(unsigned)cdiv(total, snb), snb, 0, st>>>(
           s.buckets, red_goff, s.nset, s.NB, s.seg, s.nseg, (uint32_t)s.split_G, (uint32_t)s.split_g, s.segA);
     launches++;
     uint32_t nin = s.nseg;

@@ -275,3 +275,41 @@ def test_small_n_autotune(lib):
         assert ctx.get_option(lib.OPT_WINDOW_BITS) == tuned
     finally:
         ctx.close()
+
+
+def test_graph_replay_small_n(lib):
+    """Small-n CUDA-graph replay (MSM_OPT_GRAPH): the graph is captured the second time the
+    same device scalar buffer is seen; overwriting the buffer's CONTENTS between replays must
+    change the result (kernels read memory at replay), a different buffer must not reuse the
+    graph, stage times of a replayed run read -1 while the total stays valid, and
+    MSM_OPT_GRAPH = 0 gives the same results through plain launches."""
+    import torch
+    name = "bn254"
+    c = CURVES[name]
+    n = 1 << 11
+    pts, es = gen_device_points(lib, name, n, 95)
+    ka = synth.scalars_range(c.r, 0, n, 96)
+    kb = synth.scalars_range(c.r, 0, n, 97)
+
+    def want(kw):
+        ks = synth.words_to_ints(kw)
+        return ec.to_output(ec.mul(sum(k * e for k, e in zip(ks, es)) % c.r, c.G, c))
+
+    wa, wb = want(ka), want(kb)
+    buf = torch.from_numpy(ka.view(np.int32)).cuda()
+    other = torch.from_numpy(kb.view(np.int32)).cuda()
+    ctx = lib.Context(name, pts, n=n)
+    try:
+        assert ctx.get_option(lib.OPT_GRAPH) == 1
+        for _ in range(3):                       # launch, capture, replay
+            assert ctx.run(buf) == wa
+        st = ctx.stats()
+        assert st["total_ms"] > 0 and st["accumulate_ms"] == -1.0
+        buf.copy_(other)                         # same pointer, new contents
+        assert ctx.run(buf) == wb
+        assert ctx.run(torch.from_numpy(ka.view(np.int32)).cuda()) == wa   # other buffer
+        ctx.set_option(lib.OPT_GRAPH, 0)
+        assert ctx.run(buf) == wb
+        assert ctx.stats()["accumulate_ms"] > 0
+    finally:
+        ctx.close()
