@@ -250,6 +250,16 @@ def test_chunked_host_scalars(lib, pre):
         assert ctx.get_option(lib.OPT_H2D_CHUNKS) == 1
     finally:
         ctx.close()
+    # two logical shards on one device, each uploading its half in 3 chunks from its own
+    # host thread and copy stream (f3 table on)
+    ctx = lib.Context(name, pts, n=n, devices=[0, 0])
+    try:
+        ctx.set_option(lib.OPT_PRECOMPUTE, pre)
+        ctx.set_option(lib.OPT_H2D_CHUNKS, 3)
+        assert ctx.run(ks_w) == want
+        assert ctx.get_option(lib.OPT_H2D_CHUNKS) == 3
+    finally:
+        ctx.close()
 
 
 def test_small_n_autotune(lib):
