@@ -27,6 +27,9 @@ constexpr uint32_t SIGN_BIT = 0x80000000u;
 #ifndef MSM_SEG_MINB
 #define MSM_SEG_MINB 1
 #endif
+#ifndef MSM_SEG_MINB_BIG
+#define MSM_SEG_MINB_BIG 1  // A/B: min resident blocks of k_bucket_segments for MNT4-753 (register cap)
+#endif
 
 template <class C>
 struct Layout {
@@ -1230,7 +1233,7 @@ DEVI void xyzz_mul_small(Xyzz<C>& R, const Xyzz<C>& A, uint32_t k, int bits) {
 // LAT: latency-mode products — chosen when the segments fill less than half a wave (small
 // n: a few warps walk the serial chains; ops_impl.cuh)
 template <class C, bool LAT = false>
-__global__ void __launch_bounds__(SEG_NT, MSM_SEG_SYNC ? 1 : MSM_SEG_MINB) k_bucket_segments(const uint32_t* __restrict__ buckets, const uint32_t* __restrict__ goff,
+__global__ void __launch_bounds__(SEG_NT, MSM_SEG_SYNC ? 1 : (C::L > 13 ? MSM_SEG_MINB_BIG : MSM_SEG_MINB)) k_bucket_segments(const uint32_t* __restrict__ buckets, const uint32_t* __restrict__ goff,
                                                          int nwin, uint32_t NB, uint32_t seg, uint32_t nseg,
                                                          uint32_t alpha, uint32_t beta,
                                                          uint32_t* __restrict__ out) {
