@@ -313,6 +313,22 @@ DEVI void fmul_impl(uint32_t* r, const uint32_t* a, const uint32_t* b) {
   fmul_cols<C, SQR, LAT, 0>(r, a, b, a2, m, 0ull, 0ull);
 }
 
+#ifndef MSM_FMUL2_SKEW
+#define MSM_FMUL2_SKEW 0  // A/B: product 2's column scan trails product 1's by this many columns
+#endif
+// Skewed interleave: while one product is in its few-term edge columns (latency-bound
+// m_K epilogues), the other is in its many-term middle columns (independent IMAD.WIDE).
+template <class C, bool SQR, int K, int D>
+DEVI void fmul2_skew_cols(uint32_t* r1, const uint32_t* a1, const uint32_t* b1, const uint32_t* a21, uint32_t* m1,
+                          u64& cA1, u64& cM1, uint32_t* r2, const uint32_t* a2, const uint32_t* b2,
+                          const uint32_t* a22, uint32_t* m2, u64& cA2, u64& cM2) {
+  constexpr int NC = 2 * C::L - 1;
+  if constexpr (K < NC) fmul_step<C, SQR, MSM_FMUL2_LAT != 0, K>(r1, a1, b1, a21, m1, cA1, cM1);
+  if constexpr (K >= D && K - D < NC) fmul_step<C, SQR, MSM_FMUL2_LAT != 0, K - D>(r2, a2, b2, a22, m2, cA2, cM2);
+  if constexpr (K + 1 < NC + D)
+    fmul2_skew_cols<C, SQR, K + 1, D>(r1, a1, b1, a21, m1, cA1, cM1, r2, a2, b2, a22, m2, cA2, cM2);
+}
+
 // r1 = a1*b1, r2 = a2*b2 (SQR: r1 = a1^2, r2 = a2^2), same contract as fmul
 template <class C, bool SQR = false>
 DEVI void fmul2(uint32_t* r1, const uint32_t* a1, const uint32_t* b1, uint32_t* r2, const uint32_t* a2, const uint32_t* b2) {
@@ -327,7 +343,12 @@ DEVI void fmul2(uint32_t* r1, const uint32_t* a1, const uint32_t* b1, uint32_t* 
 #pragma unroll
     for (int i = 0; i < L; i++) { d1[i] = a1[i] << 1; d2[i] = a2[i] << 1; }
   }
-  fmul2_cols<C, SQR, 0>(r1, a1, b1, d1, m1, 0ull, 0ull, r2, a2, b2, d2, m2, 0ull, 0ull);
+  if constexpr (MSM_FMUL2_SKEW > 0 && C::L <= 13) {
+    u64 cA1 = 0, cM1 = 0, cA2 = 0, cM2 = 0;
+    fmul2_skew_cols<C, SQR, 0, MSM_FMUL2_SKEW>(r1, a1, b1, d1, m1, cA1, cM1, r2, a2, b2, d2, m2, cA2, cM2);
+  } else {
+    fmul2_cols<C, SQR, 0>(r1, a1, b1, d1, m1, 0ull, 0ull, r2, a2, b2, d2, m2, 0ull, 0ull);
+  }
 }
 
 template <class C>
