@@ -588,7 +588,7 @@ def main():
                           "peak_basis": "MEASURED_PEAKS.json hbm_gbs (copy bandwidth)"},
         "stages_ms": {k: round(v, 3) for k, v in st.items() if k.endswith("_ms") and k != "table_ms"},
         "latency_ms": {"mean": ms, "min": min(times), "max": max(times)},
-        "roofline": {"kernel": "k_accumulate_sync" if L <= 13 else "k_accumulate", "bound": "alu",
+        "roofline": {"kernel": "k_accumulate_sync", "bound": "alu",
                      "achieved": achieved / 1e12, "peak": peak_imad / 1e12, "unit": "T IMAD/s",
                      "frac": achieved / peak_imad, "traffic": ncu_traffic(curve, args.log2n),
                      "work": f"{pacc} PACC x 10 field mults x (4*{L32}^2+{L32} = {4 * L32 * L32 + L32}) IMAD "

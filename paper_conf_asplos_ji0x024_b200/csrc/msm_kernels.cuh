@@ -599,7 +599,10 @@ DEVI bool point_for_entry(uint32_t* x, uint32_t* y, const uint32_t* __restrict__
 #define MSM_ACC_SYNC 1  // k_accumulate_sync (256-thread blocks in per-iteration lockstep) for L <= 13
 #endif
 #ifndef MSM_ACC_SYNC_ALL
-#define MSM_ACC_SYNC_ALL 0  // A/B: lockstep accumulation for MNT4-753 too (L1 prefetch there)
+// lockstep accumulation for MNT4-753 too (L1 prefetch there): r01 measured it slower
+// (253.7 vs 249.0 ms); in r02, after the small-n block spreading and the reduce changes,
+// it is faster — accumulate 240.2 -> 228.2 ms, C5 279.2 -> 267.9 ms
+#define MSM_ACC_SYNC_ALL 1
 #endif
 #ifndef MSM_SEG_SYNC
 #define MSM_SEG_SYNC 0  // A/B: k_bucket_segments with 256-thread blocks in per-bucket lockstep

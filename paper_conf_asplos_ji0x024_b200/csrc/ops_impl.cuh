@@ -46,7 +46,7 @@ struct Ops final : CurveOps {
     dfree(s.binCount); dfree(s.binOff); dfree(s.binCursor); dfree(s.binIdx); dfree(s.binFine);
     dfree(s.nlong); dfree(s.longs);
     dfree(s.s3Count); dfree(s.s3Off); dfree(s.s3Cursor); dfree(s.s3Sub);
-    dfree(s.s3SubCount); dfree(s.s3SubCursor); dfree(s.s3Tiles);
+    dfree(s.s3SubCount); dfree(s.s3SubCursor); dfree(s.s3Tiles); dfree(s.s3Big);
     dfree(s.s3k1); dfree(s.s3v1); dfree(s.s3k2); dfree(s.s3v2);
     dfree(s.s4Count); dfree(s.s4Off); dfree(s.s4Cursor); dfree(s.s4k); dfree(s.s4v);
     dfree(s.c4); dfree(s.goff4); dfree(s.cursor4); dfree(s.out4); dfree(s.baff_scratch);
@@ -226,6 +226,7 @@ struct Ops final : CurveOps {
       dalloc(&s.s3SubCount, NC1 * NC2);
       dalloc(&s.s3SubCursor, NC1 * NC2);
       dalloc(&s.s3Tiles, NC1 + 1);
+      dalloc(&s.s3Big, NC1 * NC2 + 1);
       dalloc(&s.s3k1, Mmax);
       dalloc(&s.s3v1, Mmax);
       dalloc(&s.s3k2, Mmax);
@@ -266,7 +267,7 @@ struct Ops final : CurveOps {
   // accumulation from chunk 1 on), so its H2D overlaps the previous chunk's work; the
   // last chunk runs the bucket reduce over every bucket (goff = nullptr) and a6.
   bool can_chunk(const Shard& s) const override {
-    return kAccSync && !s.baff && (s.sort_mode == 3 || s.sort_mode == 4) && MSM_ACC_SMEM == 0;
+    return kAccSync && C::L <= 13 && !s.baff && (s.sort_mode == 3 || s.sort_mode == 4) && MSM_ACC_SMEM == 0;
   }
   int enqueue_chunk(Shard& s, const uint32_t* scal, size_t n, size_t ibase, bool first, bool last, bool timed) override {
     if (first) CK(cudaMemsetAsync(s.buckets, 0, s.F * XW_ * sizeof(uint32_t), s.stream));
@@ -351,9 +352,13 @@ struct Ops final : CurveOps {
         k_s3_part2<uint32_t><<<maxTiles, S3_THREADS, 2 * S3_TILE * 4, st>>>(s.s3Tiles, s.s3Off, NC1, s.s3_b3, NC2, s.s3k1,
                                                                             s.s3v1, s.s3SubCursor, k2s, s.s3v2);
       CK(cudaMemcpyAsync(s.goff + s.F, s.s3Off + NC1, 4, cudaMemcpyDeviceToDevice, st));
+      CK(cudaMemsetAsync(s.s3Big, 0, sizeof(uint32_t), st));
       k_s3_part3<<<(unsigned)nsub, 256, (S3_CAP + (1u << s.s3_b3)) * 4, st>>>(s.s3Sub, s.s3_b3, (uint32_t)s.F, k2s,
-                                                                             s.s3v2, s.goff, s.sorted);
-      launches += 7;
+                                                                             s.s3v2, s.goff, s.sorted, s.cursor, s.s3Big);
+      k_s3_big_count<<<(unsigned)(2 * s.sms), 256, 0, st>>>(s.s3Sub, s.s3_b3, k2s, s.cursor, s.s3Big);
+      k_s3_big_scan<<<(unsigned)s.sms, 256, 0, st>>>(s.s3Sub, s.s3_b3, (uint32_t)s.F, s.cursor, s.s3Big, s.goff);
+      k_s3_big<<<(unsigned)(2 * s.sms), 256, 0, st>>>(s.s3Sub, s.s3_b3, k2s, s.s3v2, s.cursor, s.s3Big, s.sorted);
+      launches += 10;
     } else if (s.sort_mode == 2) {
       CK(cudaMemsetAsync(s.binCount, 0, s.FB * sizeof(uint32_t), st));
       const unsigned tiles = (unsigned)cdiv(std::max<size_t>(n, 1), BIN_TILE);
@@ -426,13 +431,17 @@ struct Ops final : CurveOps {
     k_accumulate_smem<C><<<(unsigned)cdiv(s.acc_threads, 128), 128, ACC_SLOTS * C::L * ACC_NT * 4, st>>>(pts, s.sorted, s.goff, (uint32_t)s.F,
 #else
     if constexpr (kAccSync) {
-      if (init)
-        k_accumulate_sync<C, false, true><<<(unsigned)cdiv(s.acc_threads, anb), anb, 0, st>>>(
-            pts, s.sorted, s.goff, (uint32_t)s.F, s.buckets, s.carry_pts, s.carry_f, s.acc_threads, s.nlong);
-      else if (s.baff)
-        k_accumulate_sync<C, true><<<(unsigned)cdiv(s.acc_threads, anb), anb, 0, st>>>(
-            acc_pts, s.sorted, acc_goff, (uint32_t)s.F, s.buckets, s.carry_pts, s.carry_f, s.acc_threads, s.nlong);
-      else
+      // (INIT and DIRECT instantiations only where they can run: each copy of this kernel
+      // is ~100 KB of code and minutes of MNT4-753 compile time)
+      if (C::L <= 13 && init) {
+        if constexpr (C::L <= 13)
+          k_accumulate_sync<C, false, true><<<(unsigned)cdiv(s.acc_threads, anb), anb, 0, st>>>(
+              pts, s.sorted, s.goff, (uint32_t)s.F, s.buckets, s.carry_pts, s.carry_f, s.acc_threads, s.nlong);
+      } else if (kBaff && s.baff) {
+        if constexpr (kBaff)
+          k_accumulate_sync<C, true><<<(unsigned)cdiv(s.acc_threads, anb), anb, 0, st>>>(
+              acc_pts, s.sorted, acc_goff, (uint32_t)s.F, s.buckets, s.carry_pts, s.carry_f, s.acc_threads, s.nlong);
+      } else
         k_accumulate_sync<C><<<(unsigned)cdiv(s.acc_threads, anb), anb, 0, st>>>(
             pts, s.sorted, s.goff, (uint32_t)s.F, s.buckets, s.carry_pts, s.carry_f, s.acc_threads, s.nlong);
     } else

@@ -91,7 +91,7 @@ struct Shard {
   int s3_k16 = 0;  // P1 keys as u16 (b2 + b3 <= 16)
   uint32_t *s3Count = nullptr, *s3Off = nullptr, *s3Cursor = nullptr, *s3Sub = nullptr,
            *s3k1 = nullptr, *s3v1 = nullptr, *s3k2 = nullptr, *s3v2 = nullptr, *s3SubCount = nullptr,
-           *s3SubCursor = nullptr, *s3Tiles = nullptr;
+           *s3SubCursor = nullptr, *s3Tiles = nullptr, *s3Big = nullptr;
   // two-pass cluster sort (sort4.cuh): bins of 2^s4_b2 flat buckets
   int s4_b2 = 0;
   uint32_t s4_NC1 = 0;

@@ -251,9 +251,13 @@ __global__ void __launch_bounds__(S3_THREADS) k_s3_part2(const uint32_t* __restr
 
 // P3: block = sub-bin q covering buckets [q << b3, (q+1) << b3) of [subOff[q], end_q);
 // writes goff for its buckets (< F) and the final values in bucket order.
+// Oversized sub-bins (> S3_CAP entries: skewed scalars, or a top window of lambda mod c
+// bits piling n entries into a few buckets) leave their scatter to k_s3_big: P3 writes their
+// bucket starts into gcur and lists them in big[1..big[0]].
 static __global__ void __launch_bounds__(256) k_s3_part3(const uint32_t* __restrict__ subOff, int b3, uint32_t F,
                                                          const uint16_t* __restrict__ keys2, const uint32_t* __restrict__ vals2,
-                                                         uint32_t* __restrict__ goff, uint32_t* __restrict__ sorted) {
+                                                         uint32_t* __restrict__ goff, uint32_t* __restrict__ sorted,
+                                                         uint32_t* __restrict__ gcur, uint32_t* __restrict__ big) {
   extern __shared__ uint32_t sm[];
   uint32_t* sval = sm;                  // [S3_CAP] staged values (bucket order)
   uint32_t* cnt = sm + S3_CAP;          // [2^b3]
@@ -261,6 +265,12 @@ static __global__ void __launch_bounds__(256) k_s3_part3(const uint32_t* __restr
   const uint32_t q = blockIdx.x;
   const uint32_t e0 = subOff[q], e1 = subOff[q + 1];  // subOff[nsub] = M
   const uint32_t nf = 1u << b3, fmask = nf - 1, fbase = q << b3;
+  if (e1 - e0 > (uint32_t)S3_CAP) {  // oversized: counted, scanned and scattered by k_s3_big_*
+    for (uint32_t i = threadIdx.x; i < nf; i += blockDim.x)
+      if (fbase + i < F) gcur[fbase + i] = 0;
+    if (threadIdx.x == 0) big[1 + atomicAdd(big, 1u)] = q;
+    return;
+  }
   for (uint32_t i = threadIdx.x; i < nf; i += blockDim.x) cnt[i] = 0;
   __syncthreads();
   s3_for_keys(keys2, e0, e1, [&](uint32_t f) { atomicAdd(cnt + (f & fmask), 1u); });
@@ -274,10 +284,101 @@ static __global__ void __launch_bounds__(256) k_s3_part3(const uint32_t* __restr
     s3_for_entries(keys2, vals2, e0, e1, [&](uint32_t f, uint32_t v) { sval[atomicAdd(cnt + (f & fmask), 1u)] = v; });
     __syncthreads();
     for (uint32_t p = threadIdx.x; p < len; p += blockDim.x) sorted[e0 + p] = sval[p];
-  } else {  // oversized sub-bin (skewed scalars): scatter straight to global
-    for (uint32_t e = e0 + threadIdx.x; e < e1; e += blockDim.x) {
-      const uint32_t f = __ldg(keys2 + e);
-      sorted[e0 + atomicAdd(cnt + (f & fmask), 1u)] = __ldg(vals2 + e);
+  }
+}
+
+// Oversized sub-bins, step 1: per-bucket counts by many blocks (chunks of S3_BIG_CH
+// entries, shared-memory histogram, one global atomic per (chunk, bucket)) into gcur.
+constexpr uint32_t S3_BIG_CH = 8192;
+static __global__ void __launch_bounds__(256) k_s3_big_count(const uint32_t* __restrict__ subOff, int b3,
+                                                             const uint16_t* __restrict__ keys2,
+                                                             uint32_t* __restrict__ gcur, const uint32_t* __restrict__ big) {
+  __shared__ uint32_t cnt[S3_MAXFINE];
+  const uint32_t nbig = big[0];
+  const uint32_t nf = 1u << b3, fmask = nf - 1;
+  uint32_t off = 0;
+  for (uint32_t t = 0; t < nbig; t++) {
+    const uint32_t q = big[1 + t];
+    const uint32_t e0 = subOff[q], e1 = subOff[q + 1], fbase = q << b3;
+    const uint32_t nch = (e1 - e0 + S3_BIG_CH - 1) / S3_BIG_CH;
+    // chunks of all listed sub-bins are dealt round-robin over the blocks (global chunk
+    // index off + ch), so many small oversized sub-bins (the f3 top window's low buckets)
+    // run in parallel instead of one after another
+    const uint32_t ch0 = (blockIdx.x + gridDim.x - off % gridDim.x) % gridDim.x;
+    off += nch;
+    for (uint32_t ch = ch0; ch < nch; ch += gridDim.x) {
+      const uint32_t c0 = e0 + ch * S3_BIG_CH, c1 = min(c0 + S3_BIG_CH, e1);
+      for (uint32_t i = threadIdx.x; i < nf; i += blockDim.x) cnt[i] = 0;
+      __syncthreads();
+      s3_for_keys(keys2, c0, c1, [&](uint32_t f) { atomicAdd(cnt + (f & fmask), 1u); });
+      __syncthreads();
+      for (uint32_t i = threadIdx.x; i < nf; i += blockDim.x)
+        if (cnt[i]) atomicAdd(gcur + fbase + i, cnt[i]);
+      __syncthreads();
+    }
+  }
+}
+
+// step 2: one block per oversized sub-bin scans its bucket counts into goff and the cursors
+static __global__ void __launch_bounds__(256) k_s3_big_scan(const uint32_t* __restrict__ subOff, int b3, uint32_t F,
+                                                            uint32_t* __restrict__ gcur, const uint32_t* __restrict__ big,
+                                                            uint32_t* __restrict__ goff) {
+  __shared__ uint32_t cnt[S3_MAXFINE], warp_sums[32];
+  const uint32_t nbig = big[0];
+  const uint32_t nf = 1u << b3;
+  for (uint32_t t = blockIdx.x; t < nbig; t += gridDim.x) {
+    const uint32_t q = big[1 + t];
+    const uint32_t e0 = subOff[q], fbase = q << b3;
+    for (uint32_t i = threadIdx.x; i < nf; i += blockDim.x) cnt[i] = fbase + i < F ? gcur[fbase + i] : 0u;
+    __syncthreads();
+    s3_block_scan(cnt, nf, warp_sums);
+    for (uint32_t i = threadIdx.x; i < nf; i += blockDim.x)
+      if (fbase + i < F) goff[fbase + i] = gcur[fbase + i] = e0 + cnt[i];
+    __syncthreads();
+  }
+}
+
+// step 3, the scatter: every block takes chunks of S3_BIG_CH entries of every listed
+// sub-bin, counts them per bucket in shared memory, reserves one range per (chunk, bucket)
+// with a global atomic on the bucket's cursor, and writes the entries there (a run per
+// bucket of the chunk: the degenerate one-bucket case writes whole chunks contiguously).
+// Was: one block counting and scattering the whole sub-bin (BLS12-377 2^24 at c = 21, ~n
+// entries in bucket 1: a 24 ms sort).
+static __global__ void __launch_bounds__(256) k_s3_big(const uint32_t* __restrict__ subOff, int b3,
+                                                       const uint16_t* __restrict__ keys2, const uint32_t* __restrict__ vals2,
+                                                       uint32_t* __restrict__ gcur, const uint32_t* __restrict__ big,
+                                                       uint32_t* __restrict__ sorted) {
+  __shared__ uint32_t cnt[S3_MAXFINE], gb[S3_MAXFINE];
+  const uint32_t nbig = big[0];
+  const uint32_t nf = 1u << b3, fmask = nf - 1;
+  uint32_t off = 0;
+  for (uint32_t t = 0; t < nbig; t++) {
+    const uint32_t q = big[1 + t];
+    const uint32_t e0 = subOff[q], e1 = subOff[q + 1];
+    const uint32_t fbase = q << b3;
+    const uint32_t nch = (e1 - e0 + S3_BIG_CH - 1) / S3_BIG_CH;
+    // chunks of all listed sub-bins are dealt round-robin over the blocks (global chunk
+    // index off + ch), so many small oversized sub-bins (the f3 top window's low buckets)
+    // run in parallel instead of one after another
+    const uint32_t ch0 = (blockIdx.x + gridDim.x - off % gridDim.x) % gridDim.x;
+    off += nch;
+    for (uint32_t ch = ch0; ch < nch; ch += gridDim.x) {
+      const uint32_t c0 = e0 + ch * S3_BIG_CH, c1 = min(c0 + S3_BIG_CH, e1);
+      for (uint32_t i = threadIdx.x; i < nf; i += blockDim.x) cnt[i] = 0;
+      __syncthreads();
+      s3_for_keys(keys2, c0, c1, [&](uint32_t f) { atomicAdd(cnt + (f & fmask), 1u); });
+      __syncthreads();
+      for (uint32_t i = threadIdx.x; i < nf; i += blockDim.x) {
+        const uint32_t h = cnt[i];
+        gb[i] = h ? atomicAdd(gcur + fbase + i, h) : 0u;
+        cnt[i] = 0;
+      }
+      __syncthreads();
+      s3_for_entries(keys2, vals2, c0, c1, [&](uint32_t f, uint32_t v) {
+        const uint32_t k = f & fmask;
+        sorted[gb[k] + atomicAdd(cnt + k, 1u)] = v;
+      });
+      __syncthreads();
     }
   }
 }

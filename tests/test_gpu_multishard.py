@@ -197,13 +197,15 @@ def test_bench_gpus2_self_launch():
         assert line["check"]["closed_form_match"] is True, split
 
 
+@pytest.mark.parametrize("sort", [3, 4])
 @pytest.mark.parametrize("kind,cbits,pre", [("equal", 13, 1), ("skewed", 16, 1), ("uniform", 8, 1),
                                             ("uniform", 16, 1), ("uniform", 12, 0)])
-def test_cluster_sort_heavy_bins(lib, kind, cbits, pre):
+def test_cluster_sort_heavy_bins(lib, kind, cbits, pre, sort):
     """Two-pass cluster sort (sort4.cuh) at n = 2^18 where bins exceed one cluster round
     (S4_CL * S4_CAP = 196 608 entries): equal / skewed scalars put every entry in a few
     buckets, c = 8 makes bins of 8 buckets holding ~2^20 entries each; the histogram sweep
-    and the rounds with running offsets must reproduce the closed form bit-exactly."""
+    and the rounds with running offsets must reproduce the closed form bit-exactly.  The
+    same inputs through the staged sort (3) exercise its oversized sub-bins (k_s3_big)."""
     name = "bls12_381"
     c = CURVES[name]
     n = 1 << 18
@@ -214,10 +216,10 @@ def test_cluster_sort_heavy_bins(lib, kind, cbits, pre):
     want = ec.to_output(ec.mul(sum(k * e for k, e in zip(ks, es)) % c.r, c.G, c))
     ctx = lib.Context(name, pts, n=n)
     try:
-        ctx.set_option(lib.OPT_SORT, 4)
+        ctx.set_option(lib.OPT_SORT, sort)
         ctx.set_option(lib.OPT_PRECOMPUTE, pre)
         ctx.set_option(lib.OPT_WINDOW_BITS, cbits)
-        assert ctx.get_option(lib.OPT_SORT) == 4
+        assert ctx.get_option(lib.OPT_SORT) == sort
         assert ctx.run(ks_w) == want
     finally:
         ctx.close()
