@@ -76,7 +76,45 @@ def main():
             msm.debug_field(name, op, a, a[::-1].copy())
         msm.debug_digits(name, 5, synth.scalars(c.r, 64, 3))
         print(f"{name}: ok", flush=True)
+    runs += round2_paths()
     print(f"sanitize driver: {runs} MSM runs, all equal to the closed form")
+
+
+def round2_paths():
+    """Round-2 kernels and host paths on BLS12-381: oversized sub-bins of the staged sort
+    (k_s3_big_count / scan / big, equal scalars: ~10 buckets of n entries each), the
+    two-pass cluster sort, chunked host-scalar upload with INIT accumulation, CUDA-graph
+    replay of a device scalar buffer, and the small-n autotune (context creation)."""
+    import torch
+    name, lg = "bls12_381", 14
+    c = CURVES[name]
+    n = 1 << lg
+    e0, d = synth.point_seeds(c.r, 99)
+    pts = torch.empty((n, 2 * L32[name]), dtype=torch.int32, device="cuda")
+    msm.gen_points(name, e0, d, n, pts)
+    es = [(e0 + i * d) % c.r for i in range(n)]
+    runs = 0
+    for kind in ("equal", "uniform"):
+        ks = synth.pattern_scalars(c.r, n, 98, kind) if kind == "equal" else synth.scalars_range(c.r, 0, n, 97)
+        want = ec.to_output(ec.mul(sum(k * e for k, e in zip(synth.words_to_ints(ks), es)) % c.r, c.G, c))
+        for cfg in (dict(sort=3, pre=0, c=6), dict(sort=4, pre=1, c=8), dict(sort=3, pre=1, c=10, chunks=3)):
+            ctx = msm.Context(name, pts, n=n)  # n = 2^14: the creation autotune runs too
+            ctx.set_option(msm.OPT_PRECOMPUTE, cfg["pre"])
+            ctx.set_option(msm.OPT_WINDOW_BITS, cfg["c"])
+            ctx.set_option(msm.OPT_SORT, cfg["sort"])
+            if "chunks" in cfg:
+                ctx.set_option(msm.OPT_H2D_CHUNKS, cfg["chunks"])
+            assert ctx.run(ks) == want, (kind, cfg)
+            runs += 1
+            ctx.close()
+        ctx = msm.Context(name, pts, n=n)
+        kd = torch.from_numpy(ks.view(np.int32)).cuda()
+        for _ in range(3):  # launch, capture, replay
+            assert ctx.run(kd) == want, (kind, "graph")
+            runs += 1
+        ctx.close()
+    print("round-2 paths: ok", flush=True)
+    return runs
 
 
 if __name__ == "__main__":
