@@ -465,18 +465,22 @@ def main():
         torch.cuda.synchronize()
         nst = max(2, min(args.steps, 5))
         t0 = time.perf_counter()
-        pending = []
+        pending, outs = [], []
         for i in range(nst):
             pending.append(ctx.submit(ks_np))
             if len(pending) == 2:
-                ctx.wait_words(pending.pop(0))
+                outs.append(ctx.wait_words(pending.pop(0)))
         while pending:
-            ctx.wait_words(pending.pop(0))
+            outs.append(ctx.wait_words(pending.pop(0)))
         e2e_ms = (time.perf_counter() - t0) * 1e3 / nst
+        # every pipelined result equals the device-resident run's (same scalars)
+        e2e_same = all(np.array_equal(np.asarray(o), np.asarray(res)) for o in outs)
         e2e = {"value": n / (e2e_ms / 1e3), "unit": "points/s", "ms_per_step": e2e_ms,
                "h2d_bytes_per_step": n * S * 4, "d2h_bytes_per_step": 2 * L32 * 4,
                "timing": f"host wall clock around {nst} pipelined msm_submit/msm_wait calls (pinned host scalars, "
-                         "each MSM's H2D overlaps the previous MSM's accumulation), per MSM"}
+                         "each MSM's H2D overlaps the previous MSM's accumulation; the first one, submitted into an "
+                         "empty pipeline, uploads in chunks), per MSM",
+               "results_equal_device_run": bool(e2e_same)}
         # single-call latency (one msm_run per MSM, pinned host scalars, H2D inside): the
         # library default uploads the scalars in growing chunks, each sorted and accumulated
         # while the next one uploads (MSM_OPT_H2D_CHUNKS); one copy before the MSM for contrast

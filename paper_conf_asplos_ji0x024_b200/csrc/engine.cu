@@ -748,19 +748,31 @@ long msm_submit(msm_context* ctx, const uint32_t* scalars) {
       CK(cudaMallocHost((void**)&ctx->h_result, MSM_MAX_INFLIGHT * (2 * L32 + 1) * 4));
     }
     const int q = (int)(ctx->next_ticket % MSM_MAX_INFLIGHT);
-    // copy stream: wait until the previous MSM's sort has consumed s.scal (EV_SORT is
-    // re-recorded by every pipeline, so this waits on the latest one), then H2D
-    CK(cudaStreamWaitEvent(ctx->copy_stream, s.ev[EV_SORT], 0));
     const size_t bytes = s.n * (size_t)ctx->ops->S() * 4;
     int src_dev = -1;
-    if (bytes && is_device_ptr(scalars, &src_dev)) order_after_legacy(src_dev, s.dev, ctx->copy_stream);
-    if (bytes) CK(cudaMemcpyAsync(s.scal, scalars + s.off * ctx->ops->S(), bytes, cudaMemcpyDefault, ctx->copy_stream));
-    CK(cudaEventRecord(ctx->ev_copied, ctx->copy_stream));
-    // compute stream: a2..a6 on the staged scalars, then finalise into result slot q
-    CK(cudaStreamWaitEvent(s.stream, ctx->ev_copied, 0));
-    CK(cudaEventRecord(s.ev[EV_START], s.stream));
-    CK(cudaMemsetAsync(s.err, 0, 4, s.stream));
-    ctx->launches = ctx->ops->enqueue_pipeline(s, s.scal, true);
+    const bool is_dev = bytes && is_device_ptr(scalars, &src_dev);
+    // an MSM submitted into an empty pipeline has no earlier MSM to hide its upload behind:
+    // it takes the chunked upload of msm_run (§6a) instead of one copy before its sort
+    const int K = (!is_dev && ctx->next_wait == ctx->next_ticket) ? h2d_chunks(ctx, s) : 1;
+    s.chunks_used = K;
+    if (K > 1) {
+      // s.scal is free: nothing is in flight (the chunks' copies follow s.stream's work)
+      CK(cudaEventRecord(s.ev[EV_START], s.stream));
+      CK(cudaMemsetAsync(s.err, 0, 4, s.stream));
+      ctx->launches = run_chunked(ctx, s, scalars + s.off * ctx->ops->S(), K, true);
+    } else {
+      // copy stream: wait until the previous MSM's sort has consumed s.scal (EV_SORT is
+      // re-recorded by every pipeline, so this waits on the latest one), then H2D
+      CK(cudaStreamWaitEvent(ctx->copy_stream, s.ev[EV_SORT], 0));
+      if (is_dev) order_after_legacy(src_dev, s.dev, ctx->copy_stream);
+      if (bytes) CK(cudaMemcpyAsync(s.scal, scalars + s.off * ctx->ops->S(), bytes, cudaMemcpyDefault, ctx->copy_stream));
+      CK(cudaEventRecord(ctx->ev_copied, ctx->copy_stream));
+      // compute stream: a2..a6 on the staged scalars, then finalise into result slot q
+      CK(cudaStreamWaitEvent(s.stream, ctx->ev_copied, 0));
+      CK(cudaEventRecord(s.ev[EV_START], s.stream));
+      CK(cudaMemsetAsync(s.err, 0, 4, s.stream));
+      ctx->launches = ctx->ops->enqueue_pipeline(s, s.scal, true);
+    }
     ctx->ops->enqueue_finalize(s.partial, 1, ctx->d_result[q], s.stream);
     ctx->launches++;
     CK(cudaEventRecord(s.ev[EV_END], s.stream));
